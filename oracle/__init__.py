@@ -1,0 +1,170 @@
+"""CPU ORACLE for "Judging a Type by Its Pointer" (ASPLOS'21) — TEST INFRASTRUCTURE.
+
+Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s cpu_baseline /
+``--impl reference`` leg may import this package. The product path
+(``paper_conf_asplos_zhangar21_b200``) never imports it, and it imports
+nothing from the product path: the two share only the seeded input generators
+in ``synth/``.
+
+The arithmetic lives in plain C++ (``oracle/*.cpp``, ordinary ``virtual``
+methods, objects from plain ``new`` in index order), compiled to
+``liboracle.so`` with ``g++ -O2 -ffp-contract=off -fopenmp``. This module is
+argument marshalling only. Every function cites its passage in ``oracle.h``.
+
+Pinned (tests/test_oracle_*.py, ``-m "not gpu"``) by: closed forms (micro
+val_i = init_i + R(t_i+1), region count ceil(log2(n/4096+1))), brute force
+(linear scan vs. Algorithm-1 tree on every edge address), round-trip
+invariants (TypePointer), Fig. 3's structural example, and an independent
+textbook Game-of-Life plus still-life/oscillator/glider invariants.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+
+import numpy as np
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+SO = os.path.join(HERE, "liboracle.so")
+SOURCES = ["alloc.cpp", "micro.cpp", "gol.cpp"]
+NOT_FOUND = 0xFFFFFFFF
+
+
+def build(force: bool = False) -> str:
+    srcs = [os.path.join(HERE, s) for s in SOURCES]
+    hdr = os.path.join(HERE, "oracle.h")
+    if not force and os.path.exists(SO):
+        newest = max(os.path.getmtime(p) for p in srcs + [hdr, __file__])
+        if os.path.getmtime(SO) >= newest:
+            return SO
+    cmd = ["g++", "-O2", "-std=c++17", "-ffp-contract=off", "-fopenmp", "-fPIC", "-shared",
+           "-o", SO] + srcs
+    subprocess.run(cmd, check=True)
+    return SO
+
+
+_lib = None
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        build()
+        L = ctypes.CDLL(SO)
+        u64p = ctypes.POINTER(ctypes.c_uint64)
+        u32p = ctypes.POINTER(ctypes.c_uint32)
+        L.oracle_region_plan.restype = ctypes.c_uint32
+        L.oracle_region_plan.argtypes = [ctypes.c_uint64, ctypes.c_uint64, u64p, ctypes.c_uint32]
+        L.oracle_build_table.restype = ctypes.c_uint32
+        L.oracle_build_table.argtypes = [u64p, u64p, u32p, ctypes.c_uint32, u64p, u64p, u32p]
+        L.oracle_coal_lookup.restype = None
+        L.oracle_coal_lookup.argtypes = [u64p, u64p, u32p, ctypes.c_uint32, u64p, ctypes.c_uint64, u32p]
+        L.oracle_tp_tag.restype = ctypes.c_uint64
+        L.oracle_tp_tag.argtypes = [ctypes.c_uint64, ctypes.c_uint32]
+        L.oracle_tp_type.restype = ctypes.c_uint32
+        L.oracle_tp_type.argtypes = [ctypes.c_uint64]
+        L.oracle_tp_strip.restype = ctypes.c_uint64
+        L.oracle_tp_strip.argtypes = [ctypes.c_uint64]
+        L.oracle_tp_vfunc.restype = ctypes.c_uint64
+        L.oracle_tp_vfunc.argtypes = [ctypes.c_uint64, u64p, ctypes.c_uint32, ctypes.c_uint32]
+        L.oracle_micro_run.restype = ctypes.c_int
+        L.oracle_micro_run.argtypes = [ctypes.c_uint64, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_void_p,
+                                       ctypes.c_uint32, ctypes.c_int, ctypes.c_void_p,
+                                       ctypes.POINTER(ctypes.c_double)]
+        L.oracle_gol_run.restype = ctypes.c_int
+        L.oracle_gol_run.argtypes = [ctypes.c_uint32, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_uint32,
+                                     ctypes.c_int, ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p,
+                                     ctypes.c_void_p, ctypes.POINTER(ctypes.c_double)]
+        L.oracle_max_threads.restype = ctypes.c_int
+        _lib = L
+    return _lib
+
+
+def _p(a: np.ndarray, ct):
+    return a.ctypes.data_as(ctypes.POINTER(ct))
+
+
+def max_threads() -> int:
+    return int(lib().oracle_max_threads())
+
+
+# ---- allocator / range table / COAL / TypePointer --------------------------
+def region_plan(count: int, init_chunk: int = 4096) -> list[int]:
+    L = lib()
+    k = L.oracle_region_plan(count, init_chunk, None, 0)
+    out = np.zeros(max(k, 1), dtype=np.uint64)
+    L.oracle_region_plan(count, init_chunk, _p(out, ctypes.c_uint64), k)
+    return [int(x) for x in out[:k]]
+
+
+def build_table(start, nbytes, types):
+    start = np.ascontiguousarray(start, dtype=np.uint64)
+    nbytes = np.ascontiguousarray(nbytes, dtype=np.uint64)
+    types = np.ascontiguousarray(types, dtype=np.uint32)
+    n = len(start)
+    ts = np.zeros(max(n, 1), np.uint64)
+    te = np.zeros(max(n, 1), np.uint64)
+    tt = np.zeros(max(n, 1), np.uint32)
+    K = lib().oracle_build_table(_p(start, ctypes.c_uint64), _p(nbytes, ctypes.c_uint64),
+                                 _p(types, ctypes.c_uint32), n, _p(ts, ctypes.c_uint64),
+                                 _p(te, ctypes.c_uint64), _p(tt, ctypes.c_uint32))
+    return ts[:K].copy(), te[:K].copy(), tt[:K].copy()
+
+
+def coal_lookup(t_start, t_end, t_type, addrs) -> np.ndarray:
+    t_start = np.ascontiguousarray(t_start, dtype=np.uint64)
+    t_end = np.ascontiguousarray(t_end, dtype=np.uint64)
+    t_type = np.ascontiguousarray(t_type, dtype=np.uint32)
+    addrs = np.ascontiguousarray(addrs, dtype=np.uint64)
+    out = np.zeros(len(addrs), dtype=np.uint32)
+    lib().oracle_coal_lookup(_p(t_start, ctypes.c_uint64), _p(t_end, ctypes.c_uint64),
+                             _p(t_type, ctypes.c_uint32), len(t_start), _p(addrs, ctypes.c_uint64),
+                             len(addrs), _p(out, ctypes.c_uint32))
+    return out
+
+
+def tp_tag(addr: int, t: int) -> int:
+    return int(lib().oracle_tp_tag(addr, t))
+
+
+def tp_type(q: int) -> int:
+    return int(lib().oracle_tp_type(q))
+
+
+def tp_strip(q: int) -> int:
+    return int(lib().oracle_tp_strip(q))
+
+
+def tp_vfunc(q: int, vtables, slots: int, func: int) -> int:
+    vt = np.ascontiguousarray(vtables, dtype=np.uint64)
+    return int(lib().oracle_tp_vfunc(q, _p(vt, ctypes.c_uint64), slots, func))
+
+
+# ---- apps -----------------------------------------------------------------
+def micro_run(types, init, T: int, reps: int, threads: int = 1):
+    """Returns (vals int32[n], seconds of the dispatch passes)."""
+    types = np.ascontiguousarray(types, dtype=np.uint32)
+    init = np.ascontiguousarray(init, dtype=np.int32)
+    n = len(types)
+    out = np.zeros(n, dtype=np.int32)
+    sec = ctypes.c_double(0.0)
+    rc = lib().oracle_micro_run(n, T, types.ctypes.data, init.ctypes.data, reps, threads,
+                                out.ctypes.data, ctypes.byref(sec))
+    if rc != 0:
+        raise ValueError(f"oracle_micro_run rc={rc}")
+    return out, sec.value
+
+
+def gol_run(W: int, H: int, alive0, gens: int, torus: bool = False, threads: int = 1):
+    """Returns (state uint8[H*W], counter uint16[H*W], pop uint32[gens], seconds)."""
+    a = np.ascontiguousarray(alive0, dtype=np.uint8)
+    st = np.zeros(W * H, np.uint8)
+    ctr = np.zeros(W * H, np.uint16)
+    pop = np.zeros(max(gens, 1), np.uint32)
+    sec = ctypes.c_double(0.0)
+    rc = lib().oracle_gol_run(W, H, a.ctypes.data, gens, int(torus), threads, st.ctypes.data,
+                              ctr.ctypes.data, pop.ctypes.data, ctypes.byref(sec))
+    if rc != 0:
+        raise ValueError(f"oracle_gol_run rc={rc}")
+    return st, ctr, pop[:gens].copy(), sec.value

@@ -1,0 +1,98 @@
+/*
+ * oracle.h — C ABI of the CPU ORACLE for "Judging a Type by Its Pointer:
+ * Optimizing GPU Virtual Functions" (Zhang, Alawneh, Rogers, ASPLOS'21).
+ *
+ * TEST INFRASTRUCTURE ONLY. Only tests/, __graft_entry__.smoke() and
+ * bench.py's cpu_baseline / --impl reference leg may load liboracle.so.
+ * It shares no code, header, table or constant generator with the CUDA path
+ * (paper_conf_asplos_zhangar21_b200/csrc, include/vf.h), and neither side
+ * includes the other.
+ *
+ * Citations are P:<line> of /root/reference/PAPER.md (section / figure /
+ * algorithm given alongside). Readings of silent or garbled passages are the
+ * G-numbers listed in DESIGN.md §"Readings".
+ *
+ * Plain, slow, obviously-correct: ordinary C++ classes with `virtual`
+ * methods, objects from plain `new`, one per object, in index order; loops in
+ * the paper's order. OpenMP (threads>1) only splits independent per-object
+ * loops; results are identical for any thread count (tested).
+ */
+#ifndef VF_ORACLE_H
+#define VF_ORACLE_H
+#include <stdint.h>
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define ORACLE_NOT_FOUND 0xFFFFFFFFu
+
+/* ---- Allocator region policy (§4; §5) ------------
+ * Capacities (in objects) of the regions SharedOA creates for one type when
+ * `count` objects are allocated: r0 = init_chunk, r_{j+1} = 2 r_j, until the
+ * sum reaches count. Returns the number of regions (0 if count == 0), writes
+ * at most max_out capacities. */
+uint32_t oracle_region_plan(uint64_t count, uint64_t init_chunk,
+                            uint64_t* caps_out, uint32_t max_out);
+
+/* ---- Virtual range table (Fig. 3) --------------
+ * Build the table from raw regions [start_i, start_i + bytes_i) of type
+ * type_i: sort by start, merge a region into its predecessor when it is of
+ * the same type and exactly adjacent. Writes K <= n rows
+ * (start, end, type); returns K. */
+uint32_t oracle_build_table(const uint64_t* start, const uint64_t* bytes,
+                            const uint32_t* type, uint32_t n,
+                            uint64_t* t_start, uint64_t* t_end, uint32_t* t_type);
+
+/* ---- COAL ObjectRangeLookup (Algorithm 1) ----
+ * Balanced segment tree over the K sorted disjoint ranges (leaves = ranges,
+ * internal nodes = [min start, max end) of their children), descended from
+ * the root; returns the type of the leaf whose [start,end) contains addr,
+ * else ORACLE_NOT_FOUND (Alg. 1 "return NULL"). Reading G5. */
+void oracle_coal_lookup(const uint64_t* t_start, const uint64_t* t_end,
+                        const uint32_t* t_type, uint32_t K,
+                        const uint64_t* addrs, uint64_t n, uint32_t* out_type);
+
+/* ---- TypePointer (Fig. 5; §6.1; §6.3)
+ * B200 format (reading G6): 7-bit tag in bits 63:57 above the 57-bit VA;
+ * tag = type+1 (0 = untagged). Pattern of the upper bits = 0 (reading G7). */
+uint64_t oracle_tp_tag(uint64_t addr, uint32_t type);
+uint32_t oracle_tp_type(uint64_t tagged);     /* ORACLE_NOT_FOUND if untagged */
+uint64_t oracle_tp_strip(uint64_t tagged);
+/* Fig. 5b with the padded-index form:
+ * vFunc = vtables[type(q) * vtable_slots + func_index]. */
+uint64_t oracle_tp_vfunc(uint64_t tagged, const uint64_t* vtables,
+                         uint32_t vtable_slots, uint32_t func_index);
+
+/* ---- Config 2 microbenchmark (§8.3) ------------------------
+ * n objects; object i is of class MObj<types[i]> (types[i] < T <= 32) with
+ * val = init[i]; `reps` passes of `for i: objs[i]->apply()` where
+ * MObj<k>::apply() { val += k + 1; } ("simple addition").
+ * out_vals[i] = final val. *seconds = wall time of the dispatch passes only.
+ * threads = OpenMP threads over i (1 = the reference semantics). */
+int oracle_micro_run(uint64_t n, uint32_t T, const uint32_t* types,
+                     const int32_t* init, uint32_t reps, int threads,
+                     int32_t* out_vals, double* seconds);
+
+/* ---- Config 1 Game of Life (Table 2; readings G12-G14) -----
+ * Grid W x H, cell c = y*W + x. Each cell owns one Alive and one Dead
+ * object; grid[c] points at the one matching its state. Per generation:
+ *  (1) n[c] = live neighbours among 8 in the previous state (dead border,
+ *      or torus if torus != 0);
+ *  (2) s' = grid[c]->next(n[c])  (virtual; Alive: n==2||n==3, Dead: n==3;
+ *      both increment their own counter: age / dead_for);
+ *  (3) if s' != s: grid[c] = the other object, whose counter is reset to 0.
+ * Outputs: final state (uint8), final counter of each cell's current object,
+ * population after every generation pop[g], g = 0..gens-1.
+ * *seconds = wall time of the generation loop. */
+int oracle_gol_run(uint32_t W, uint32_t H, const uint8_t* init_alive,
+                   uint32_t gens, int torus, int threads,
+                   uint8_t* out_state, uint16_t* out_counter, uint32_t* pop,
+                   double* seconds);
+
+/* number of OpenMP threads actually available */
+int oracle_max_threads(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif
