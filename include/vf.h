@@ -1,0 +1,232 @@
+/*
+ * vf.h — C ABI of libvf.so: B200-native GPU virtual-function dispatch after
+ * "Judging a Type by Its Pointer: Optimizing GPU Virtual Functions"
+ * (Zhang, Alawneh, Rogers, ASPLOS'21). Citations are P:<line> of the paper
+ * text with the section / figure / algorithm they fall in.
+ *
+ * The paper's user-visible operations are
+ *   - `Obj* = sharedNew TYPE()`                 (Fig. 4, §4)
+ *       -> vf_alloc_typed / vf_alloc_typed_batch (type-based arenas + the
+ *          virtual range table of Fig. 3)
+ *   - device `new TYPE()` of the CUDA baseline
+ *       -> vf_alloc_cuda
+ *   - TypePointer `new` returning a tagged pointer (Fig. 5a P:1178-1180,
+ *       §6.1) -> `tag` = 1 on any allocation call
+ *   - `obj->vFun()` (Fig. 4) resolved four ways:
+ *       vf_dispatch_cuda      embedded vTable* -> vFunc* -> indirect CALL
+ *                             (Fig. 1a, §2)
+ *       vf_dispatch_sharedoa  the same call on SharedOA-allocated objects (§4)
+ *       vf_dispatch_coal      ObjectRangeLookup on the object address alone
+ *                             (§5, Algorithm 1)
+ *       vf_dispatch_typeptr   type from the pointer's upper bits (§6, Fig. 5b)
+ *
+ * Conventions (all functions):
+ *   - extern "C", never throw; return vf_status (VF_OK == 0). On failure a
+ *     human-readable detail is available from vf_last_error(ctx).
+ *   - Pointer arguments named *_dev are DEVICE pointers (caller-owned, e.g.
+ *     torch tensors' data_ptr()); all others are host pointers.
+ *   - All device work is enqueued on `stream` (a cudaStream_t passed as
+ *     void*; NULL = legacy default stream) and is asynchronous; CUDA faults
+ *     surface on a later call as VF_ERR_CUDA.
+ *   - A ctx is bound to one device and must not be used from two host
+ *     threads at once. Type ids are app-local (0 .. ntypes-1) and global
+ *     across ranks; addresses and range tables are per device.
+ *   - Ownership: the ctx owns every object, arena, range table and the
+ *     device heap objects it created; the caller owns pointer arrays,
+ *     argument blobs and output buffers.
+ */
+#ifndef VF_H
+#define VF_H
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  VF_OK = 0,
+  VF_ERR_INVALID = 1,         /* bad argument (null ctx, unknown app/method/type, ...) */
+  VF_ERR_OOM = 2,             /* device memory / device heap / VA exhausted            */
+  VF_ERR_CUDA = 3,            /* a CUDA runtime/driver call failed                     */
+  VF_ERR_TAG_BITS = 4,        /* an object address has bits 63:57 != 0  */
+  VF_ERR_TOO_MANY_TYPES = 5,  /* more types than a 7-bit tag / 32-lane group can hold  */
+  VF_ERR_TABLE_FULL = 6,      /* range table larger than VF_MAX_RANGES                 */
+  VF_ERR_UNSUPPORTED = 7      /* valid but not implemented for this app/variant        */
+} vf_status;
+
+typedef enum { VF_CUDA = 0, VF_SHAREDOA = 1, VF_COAL = 2, VF_TYPEPTR = 3 } vf_variant;
+
+/* Workload apps compiled into libvf.so (GPUs cannot load code at run time,
+ * so every class whose virtual methods a kernel may call is compiled into
+ * that kernel's module: P:607-615). */
+enum {
+  VF_APP_MICRO = 0, /* config 2: MObj<k>::apply(){ val += k+1; }  (§8.3)      */
+  VF_APP_GOL = 1,   /* config 1: Cell / Alive / Dead               (Table 2)  */
+  VF_APP_COUNT = 2
+};
+
+/* Methods of VF_APP_MICRO (args structs are passed by value, see dispatch). */
+enum { VF_MICRO_APPLY = 0, /* args: none                                       */
+       VF_MICRO_GET = 1 }; /* args: vf_micro_get_args — out_dev[i] = objs[i].val */
+typedef struct { int32_t* out_dev; } vf_micro_get_args;
+
+/* Methods of VF_APP_GOL. */
+enum { VF_GOL_NEXT = 0, /* args: vf_gol_next_args (one generation, step 2 of W1) */
+       VF_GOL_GET = 1 };/* args: vf_gol_get_args                                  */
+typedef struct {
+  const uint8_t* nbr_dev;   /* live-neighbour count per cell (cell id = object's own index) */
+  uint8_t* state_out_dev;   /* next state per cell                                          */
+} vf_gol_next_args;
+typedef struct { uint16_t* counter_out_dev; uint8_t* type_out_dev; } vf_gol_get_args;
+
+#define VF_MAX_RANGES 4096u     /* COAL range-table capacity (staged in shared memory)   */
+#define VF_MAX_ARGS_BYTES 256u  /* method argument blob, copied into kernel parameters   */
+#define VF_VA_BITS 57u          /* TypePointer: tag in bits 63:57 (reading G6)           */
+#define VF_NOT_FOUND 0xFFFFFFFFu
+
+typedef struct vf_ctx vf_ctx;
+
+typedef struct {
+  int device;                /* CUDA device ordinal                                        */
+  uint64_t init_chunk_objs;  /* first region size in objects (4K)               */
+  int reserve_va;            /* 1: reserve one VA window per type so consecutive regions   */
+                             /*    are contiguous and merge (K = #types); 0: one           */
+                             /*    cudaMalloc per region (K grows as log2)      */
+  uint64_t va_window_bytes;  /* VA reserved per (app,type) when reserve_va (default 64 GiB)*/
+  uint64_t cuda_heap_bytes;  /* device malloc heap for vf_alloc_cuda; must   */
+                             /* be set before any device-malloc kernel in the process      */
+} vf_config;
+
+/* One row of the virtual range table (Fig. 3): [start, end) holds objects of
+ * (app, type_id) whose embedded device vTable* equals vptr. Reading G1:
+ * "Range" is the end address, half-open. */
+typedef struct {
+  uint64_t start, end;
+  uint32_t type_id, app;
+  uint64_t vptr;
+} vf_range;
+
+/* One raw allocator region before merging. */
+typedef struct {
+  uint64_t start;
+  uint64_t cap_objs;   /* capacity in objects (4096, 8192, ... per type)  */
+  uint64_t used_objs;
+  uint32_t obj_bytes;  /* stride = sizeof(class)                          */
+  uint32_t type_id, app, pad;
+} vf_region;
+
+/* Fills *cfg with defaults: device 0, 4096, reserve_va 1, 64 GiB, 8 GiB heap. */
+void vf_config_default(vf_config* cfg);
+vf_status vf_create(const vf_config* cfg, vf_ctx** out);
+/* Frees all arenas and device-heap objects; every object pointer becomes invalid. */
+void vf_destroy(vf_ctx* ctx);
+const char* vf_status_str(vf_status s);
+const char* vf_last_error(const vf_ctx* ctx);
+
+/* App metadata: number of concrete types, sizeof each type (bytes, ntypes
+ * entries written to obj_bytes if non-null), number of methods. */
+vf_status vf_app_info(uint32_t app, uint32_t* ntypes, uint32_t* obj_bytes, uint32_t* nmethods);
+
+/* ---- allocation (one-time; not timed) --------- */
+/* `count` objects of class (app, type_id), placed at the next slots of that
+ * type's arena (regions of 4K, 8K, ... objects) and constructed on
+ * the device (vTable* installed). ctor_args_dev: optional
+ * per-object constructor argument blob (ctor_arg_bytes each, app-defined,
+ * may be NULL). Writes `count` u64 pointers to out_ptrs_dev. tag = 1 returns
+ * TypePointer pointers: (type_id+1) << 57 | address (Fig. 5a). Objects live
+ * until vf_reset / vf_destroy. */
+vf_status vf_alloc_typed(vf_ctx* ctx, uint32_t app, uint32_t type_id, uint64_t count,
+                         const void* ctor_args_dev, uint32_t ctor_arg_bytes,
+                         uint64_t* out_ptrs_dev, int tag, void* stream);
+/* Batched: object i is of class (app, type_ids_dev[i]) and takes the next
+ * slot of its type's arena in index order (allocation order = index order). */
+vf_status vf_alloc_typed_batch(vf_ctx* ctx, uint32_t app, const uint32_t* type_ids_dev,
+                               uint64_t count, const void* ctor_args_dev,
+                               uint32_t ctor_arg_bytes, uint64_t* out_ptrs_dev, int tag,
+                               void* stream);
+/* CUDA baseline: device-heap `new` of class (app, type_ids_dev[i]) per object
+ * in a kernel. tag = 1 additionally tags the
+ * returned pointers (TypePointer on the default CUDA allocator, §8.2
+ * P:2749-2757); such objects are NOT in the range table. */
+vf_status vf_alloc_cuda(vf_ctx* ctx, uint32_t app, const uint32_t* type_ids_dev, uint64_t count,
+                        const void* ctor_args_dev, uint32_t ctor_arg_bytes,
+                        uint64_t* out_ptrs_dev, int tag, void* stream);
+/* Drop every object (arenas unmapped, device-heap objects deleted); VA
+ * reservations are kept. Synchronises the device. */
+vf_status vf_reset(vf_ctx* ctx);
+
+/* Sorted, disjoint, merged range table of `app` (app = 0xFFFFFFFF: all
+ * apps). Host view owned by ctx, valid until the next alloc / reset. */
+vf_status vf_range_table(const vf_ctx* ctx, uint32_t app, const vf_range** out, uint32_t* n);
+/* Raw regions in creation order (owned by ctx, same lifetime). */
+vf_status vf_regions(const vf_ctx* ctx, const vf_region** out, uint32_t* n);
+/* Device vTable* of each concrete type of `app` (ntypes entries, host array). */
+vf_status vf_type_vptrs(vf_ctx* ctx, uint32_t app, uint64_t* vptrs_out);
+
+/* ---- resolution / verification ---------------------------------------- */
+/* types_out_dev[i] = type id of ptrs_dev[i] under the variant's rule
+ * (CUDA/SHAREDOA: embedded vTable* -> type; COAL: range lookup; TYPEPTR:
+ * tag); VF_NOT_FOUND if unresolved (the dispatch kernels fall back to the
+ * embedded vTable* for those) or if the pointer is null. */
+vf_status vf_resolve(vf_ctx* ctx, uint32_t app, vf_variant v, const uint64_t* ptrs_dev,
+                     uint64_t n, uint32_t* types_out_dev, void* stream);
+/* Brute-force type identity: counts pointers whose variant-resolved type's
+ * vTable* differs from the vTable* embedded in the object (or that fail to
+ * resolve). Adds the count to *mismatches_dev (u64, device). */
+vf_status vf_verify_types(vf_ctx* ctx, uint32_t app, vf_variant v, const uint64_t* ptrs_dev,
+                          uint64_t n, unsigned long long* mismatches_dev, void* stream);
+
+/* ---- dispatch: one call of virtual method `method` on every objs_dev[i],
+ * i in [0, n); null entries are skipped. `args` is a host pointer to the
+ * method's argument struct (args_bytes <= VF_MAX_ARGS_BYTES), copied into
+ * the kernel parameters. Pointers must be unique for mutating methods.
+ * CUDA / SHAREDOA: plain C++ virtual call (vTable* load, vFunc* load,
+ * indirect CALL). COAL: range lookup in shared memory. TYPEPTR: tag shift +
+ * strip. COAL and TYPEPTR then group the lanes of a warp by type and run
+ * each type's body once per warp as a direct, inlined call. */
+vf_status vf_dispatch_cuda(vf_ctx* ctx, uint32_t app, uint32_t method, const uint64_t* objs_dev,
+                           uint64_t n, const void* args, size_t args_bytes, void* stream);
+vf_status vf_dispatch_sharedoa(vf_ctx* ctx, uint32_t app, uint32_t method,
+                               const uint64_t* objs_dev, uint64_t n, const void* args,
+                               size_t args_bytes, void* stream);
+vf_status vf_dispatch_coal(vf_ctx* ctx, uint32_t app, uint32_t method, const uint64_t* objs_dev,
+                           uint64_t n, const void* args, size_t args_bytes, void* stream);
+vf_status vf_dispatch_typeptr(vf_ctx* ctx, uint32_t app, uint32_t method,
+                              const uint64_t* objs_dev, uint64_t n, const void* args,
+                              size_t args_bytes, void* stream);
+/* Same, variant as a parameter. */
+vf_status vf_dispatch(vf_ctx* ctx, vf_variant v, uint32_t app, uint32_t method,
+                      const uint64_t* objs_dev, uint64_t n, const void* args, size_t args_bytes,
+                      void* stream);
+
+/* ---- app helpers (non-virtual phases) ---------------------------------- */
+/* GOL step (1): nbr_dev[c] = live neighbours of cell c in state_dev (W x H,
+ * dead border, or torus if torus != 0). */
+vf_status vf_gol_neighbors(uint32_t W, uint32_t H, int torus, const uint8_t* state_dev,
+                           uint8_t* nbr_dev, void* stream);
+/* GOL step (3): where state_next != state_prev, swap grid_dev[c] between
+ * alive_dev[c] and dead_dev[c] and reset the new object's counter. */
+vf_status vf_gol_swap(vf_ctx* ctx, uint64_t ncells, const uint8_t* state_prev_dev,
+                      const uint8_t* state_next_dev, uint64_t* grid_dev,
+                      const uint64_t* alive_dev, const uint64_t* dead_dev, void* stream);
+
+/* ---- utilities ---------------------------------------------------------- */
+/* sum over i of vals_dev[i] (int32, widened) into *out_dev (i64, device). */
+vf_status vf_checksum_i32(const int32_t* vals_dev, uint64_t n, long long* out_dev, void* stream);
+/* Benchmark / ablation knobs of the COAL / TYPEPTR kernels (process-wide):
+ * "unroll" = objects per thread (1, 2, 4; -1 = app default), "prefetch" =
+ * 1/0 to issue (or not) an L1 prefetch of every object line before the type
+ * groups run (-1 = default on). VF_ERR_INVALID for unknown keys / values. */
+vf_status vf_set_tuning(const char* key, int value);
+/* Number of libvf kernel launches issued since load (for bench accounting). */
+uint64_t vf_launch_count(void);
+
+/* Strip a TypePointer tag (restore the upper bits before any
+ * field access). Host-side helper; the kernels do the same with one LOP3. */
+static inline uint64_t vf_strip(uint64_t p) { return p & ((1ull << VF_VA_BITS) - 1); }
+
+#ifdef __cplusplus
+}
+#endif
+#endif

@@ -1,0 +1,112 @@
+"""Workload drivers over the C ABI (argument marshalling and step sequencing only).
+
+Each driver allocates its objects through libvf (typed arenas for sharedoa /
+coal / typeptr, device-heap `new` for cuda), then a `step()` enqueues the
+app's kernels on a stream. Inputs come from ``synth`` (seeded; shared with the
+oracle tests); nothing here computes any part of the method.
+"""
+from __future__ import annotations
+
+import numpy as np
+import torch
+
+import synth
+
+from . import vf
+
+
+def _dev(device):
+    return torch.device(f"cuda:{device}" if isinstance(device, int) else device)
+
+
+class Micro:
+    """Config 2: one virtual `apply()` per object over n objects of T types.
+
+    Paper §8.3. Object i has type t(i) (synth.micro_types) and
+    val = init_i; after R steps val_i = init_i + R (t(i)+1).
+    """
+
+    def __init__(self, ctx: vf.Ctx, n: int, T: int, order: str = "random", seed: int = 42,
+                 variant: str = "typeptr", k: int | None = None, types_np=None, init_np=None):
+        self.ctx, self.n, self.T, self.variant = ctx, n, T, variant
+        self.v = vf.VARIANTS[variant]
+        dev = _dev(ctx.device)
+        if types_np is None:
+            types_np = synth.micro_types(n, T, order, seed=seed, k=k)
+        if init_np is None:
+            init_np = synth.micro_init(n, seed=seed)
+        self.types = torch.from_numpy(types_np.astype(np.int32)).to(dev)
+        init = torch.from_numpy(init_np.astype(np.int32)).to(dev)
+        if variant == "cuda":
+            self.objs = ctx.alloc_cuda(vf.APP_MICRO, self.types, init)
+        else:
+            self.objs = ctx.alloc_typed_batch(vf.APP_MICRO, self.types, init, tag=(variant == "typeptr"))
+        torch.cuda.synchronize(dev)
+        self._ptr = int(self.objs.data_ptr())
+
+    def step(self, stream=None):
+        st = self.ctx.dispatch_raw(self.v, vf.APP_MICRO, vf.MICRO_APPLY, self._ptr, self.n, None,
+                                   vf._stream(stream))
+        if st:
+            self.ctx._check(st, "micro step")
+
+    def values(self, out=None, stream=None):
+        if out is None:
+            out = torch.empty(self.n, dtype=torch.int32, device=self.objs.device)
+        self.ctx.dispatch(self.v, vf.APP_MICRO, vf.MICRO_GET, self.objs,
+                          vf.micro_get_args(out.data_ptr()), stream=stream)
+        return out
+
+
+class Gol:
+    """Config 1: Game of Life over polymorphic Alive / Dead cells (Table 2).
+
+    Per generation: (1) vf_gol_neighbors, (2) one virtual next() per
+    cell, (3) vf_gol_swap. Every cell owns one object in each type's arena, so
+    a type change is a pointer swap.
+    """
+
+    def __init__(self, ctx: vf.Ctx, W: int, H: int, alive0, variant: str = "typeptr",
+                 torus: bool = False):
+        self.ctx, self.W, self.H, self.variant, self.torus = ctx, W, H, variant, torus
+        self.v = vf.VARIANTS[variant]
+        dev = _dev(ctx.device)
+        N = W * H
+        self.N = N
+        cells = torch.arange(N, dtype=torch.int32, device=dev)
+        if variant == "cuda":
+            self.alive = ctx.alloc_cuda(vf.APP_GOL, torch.ones(N, dtype=torch.int32, device=dev), cells)
+            self.dead = ctx.alloc_cuda(vf.APP_GOL, torch.zeros(N, dtype=torch.int32, device=dev), cells)
+        else:
+            tag = variant == "typeptr"
+            self.alive = ctx.alloc_typed(vf.APP_GOL, 1, N, cells, tag=tag)
+            self.dead = ctx.alloc_typed(vf.APP_GOL, 0, N, cells, tag=tag)
+        self.grid = self.dead.clone()
+        a0 = torch.from_numpy(np.ascontiguousarray(alive0, dtype=np.uint8)).to(dev)
+        zeros = torch.zeros(N, dtype=torch.uint8, device=dev)
+        vf.gol_swap(ctx, zeros, a0, self.grid, self.alive, self.dead)  # grid <- initial types
+        self.state = a0.clone()
+        self.next = torch.empty_like(self.state)
+        self.nbr = torch.empty_like(self.state)
+        self.args = [vf.gol_next_args(self.nbr.data_ptr(), self.next.data_ptr()),
+                     vf.gol_next_args(self.nbr.data_ptr(), self.state.data_ptr())]
+        self.parity = 0
+        torch.cuda.synchronize(dev)
+
+    def gen(self, stream=None):
+        cur, nxt = (self.state, self.next) if self.parity == 0 else (self.next, self.state)
+        vf.gol_neighbors(self.W, self.H, cur, self.nbr, self.torus, stream)
+        self.ctx.dispatch(self.v, vf.APP_GOL, vf.GOL_NEXT, self.grid, self.args[self.parity], stream=stream)
+        vf.gol_swap(self.ctx, cur, nxt, self.grid, self.alive, self.dead, stream)
+        self.parity ^= 1
+
+    @property
+    def current(self):
+        return self.state if self.parity == 0 else self.next
+
+    def counters(self):
+        ctr = torch.empty(self.N, dtype=torch.int16, device=self.grid.device)
+        typ = torch.empty(self.N, dtype=torch.uint8, device=self.grid.device)
+        self.ctx.dispatch(self.v, vf.APP_GOL, vf.GOL_GET, self.grid,
+                          vf.gol_get_args(ctr.data_ptr(), typ.data_ptr()))
+        return ctr, typ

@@ -1,0 +1,718 @@
+// core.cu — host side of libvf.so: context, the type-based arena allocator
+// (SharedOA, §4), the virtual range table (Fig. 3), TypePointer
+// tagging (§6.1), and the C-ABI entry points declared in include/vf.h.
+//
+// B200 design: device memory only (no UVM objects, SURVEY A7 OUT). With
+// reserve_va = 1 each (app, type) gets one reserved VA window
+// (cuMemAddressReserve) and its doubling regions are mapped
+// back-to-back inside it, so the paper's "merge contiguous regions" always
+// fires and the COAL table has exactly one row per type. With reserve_va = 0
+// every region is its own cudaMalloc and the table grows as
+// T * ceil(log2(n/4096 + 1)) rows, reproducing the fragmented case.
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <atomic>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <map>
+#include <string>
+#include <vector>
+
+#include "vf_internal.h"
+
+namespace vf {
+static std::atomic<uint64_t> g_launches{0};
+void note_launch(uint64_t k) { g_launches.fetch_add(k, std::memory_order_relaxed); }
+Tuning& tuning() {
+  static Tuning t;
+  return t;
+}
+
+static const AppOps* app_ops(uint32_t app) {
+  switch (app) {
+    case VF_APP_MICRO: return app_micro();
+    case VF_APP_GOL: return app_gol();
+  }
+  return nullptr;
+}
+
+// ---- driver entry points (no link-time dependency on libcuda) -------------
+struct Drv {
+  decltype(&cuMemAddressReserve) reserve = nullptr;
+  decltype(&cuMemAddressFree) addr_free = nullptr;
+  decltype(&cuMemCreate) create = nullptr;
+  decltype(&cuMemRelease) release = nullptr;
+  decltype(&cuMemMap) map = nullptr;
+  decltype(&cuMemUnmap) unmap = nullptr;
+  decltype(&cuMemSetAccess) set_access = nullptr;
+  decltype(&cuMemGetAllocationGranularity) granularity = nullptr;
+  bool ok = false;
+};
+
+template <class F>
+static bool get_entry(const char* name, F& f) {
+  void* p = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  if (cudaGetDriverEntryPoint(name, &p, cudaEnableDefault, &q) != cudaSuccess ||
+      q != cudaDriverEntryPointSuccess || !p)
+    return false;
+  f = reinterpret_cast<F>(p);
+  return true;
+}
+
+static Drv& drv() {
+  static Drv d;
+  static bool init = false;
+  if (!init) {
+    init = true;
+    d.ok = get_entry("cuMemAddressReserve", d.reserve) && get_entry("cuMemAddressFree", d.addr_free) &&
+           get_entry("cuMemCreate", d.create) && get_entry("cuMemRelease", d.release) &&
+           get_entry("cuMemMap", d.map) && get_entry("cuMemUnmap", d.unmap) &&
+           get_entry("cuMemSetAccess", d.set_access) &&
+           get_entry("cuMemGetAllocationGranularity", d.granularity);
+  }
+  return d;
+}
+
+struct Arena {
+  uint32_t app = 0, type = 0, obj_bytes = 0;
+  uint64_t next_cap = 0;     // capacity (objects) of the next region
+  int cur = -1;              // current region (index into ctx->regions)
+  uint64_t used_bytes = 0;   // VMM: bytes of the window covered by regions
+  CUdeviceptr va = 0;        // VMM window
+  uint64_t va_size = 0;
+  uint64_t mapped = 0;       // VMM: bytes mapped from the window start
+  std::vector<CUmemGenericAllocationHandle> handles;
+  std::vector<std::pair<CUdeviceptr, size_t>> maps;
+};
+
+struct AppTable {
+  std::vector<vf_range> rows;
+  uint64_t* d_start = nullptr;
+  uint64_t* d_end = nullptr;
+  uint32_t* d_type = nullptr;
+  uint32_t d_cap = 0;
+  uint32_t K = 0, P = 1;
+  std::vector<uint64_t> vptr;
+  uint64_t* d_vptr = nullptr;
+  bool vptr_ready = false;
+};
+
+struct HeapBatch {
+  uint32_t app;
+  uint64_t* d_ptrs;  // untagged pointers, for delete
+  uint64_t n;
+};
+}  // namespace vf
+
+using namespace vf;
+
+struct vf_ctx {
+  vf_config cfg;
+  std::string err;
+  std::map<std::pair<uint32_t, uint32_t>, Arena> arenas;
+  std::vector<vf_region> regions;
+  std::vector<void*> region_malloc;  // non-VMM: cudaMalloc base per region (else null)
+  std::vector<vf_range> all_rows;
+  AppTable tables[VF_APP_COUNT];
+  std::vector<HeapBatch> heap;
+  std::vector<uint64_t> type_count[VF_APP_COUNT];  // live objects per (app, type)
+  size_t gran = 2u << 20;
+};
+
+namespace {
+
+vf_status fail(vf_ctx* c, vf_status s, const char* fmt, ...) {
+  if (c) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    c->err = buf;
+  }
+  return s;
+}
+
+#define CUDA_TRY(ctx, call)                                                                  \
+  do {                                                                                       \
+    cudaError_t _e = (call);                                                                 \
+    if (_e != cudaSuccess)                                                                   \
+      return fail(ctx, VF_ERR_CUDA, "%s: %s (%s:%d)", #call, cudaGetErrorString(_e), __FILE__, \
+                  __LINE__);                                                                 \
+  } while (0)
+
+#define DRV_TRY(ctx, call)                                                                     \
+  do {                                                                                         \
+    CUresult _r = (call);                                                                      \
+    if (_r != CUDA_SUCCESS)                                                                    \
+      return fail(ctx, _r == CUDA_ERROR_OUT_OF_MEMORY ? VF_ERR_OOM : VF_ERR_CUDA,             \
+                  "%s: CUresult %d (%s:%d)", #call, (int)_r, __FILE__, __LINE__);              \
+  } while (0)
+
+inline cudaStream_t S(void* s) { return reinterpret_cast<cudaStream_t>(s); }
+
+uint64_t round_up(uint64_t x, uint64_t g) { return (x + g - 1) / g * g; }
+
+vf_status set_device(vf_ctx* c) {
+  CUDA_TRY(c, cudaSetDevice(c->cfg.device));
+  return VF_OK;
+}
+
+// Ensure the (app,type) arena has a VA window (VMM mode).
+vf_status ensure_window(vf_ctx* c, Arena& a) {
+  if (a.va) return VF_OK;
+  Drv& d = drv();
+  if (!d.ok) return fail(c, VF_ERR_UNSUPPORTED, "CUDA VMM driver entry points unavailable");
+  a.va_size = round_up(c->cfg.va_window_bytes, c->gran);
+  DRV_TRY(c, d.reserve(&a.va, a.va_size, c->gran, 0, 0));
+  return VF_OK;
+}
+
+vf_status map_upto(vf_ctx* c, Arena& a, uint64_t need_bytes) {
+  if (need_bytes <= a.mapped) return VF_OK;
+  if (need_bytes > a.va_size)
+    return fail(c, VF_ERR_OOM, "type window of %llu bytes exhausted (need %llu)",
+                (unsigned long long)a.va_size, (unsigned long long)need_bytes);
+  Drv& d = drv();
+  const uint64_t sz = round_up(need_bytes - a.mapped, c->gran);
+  CUmemAllocationProp prop = {};
+  prop.type = CU_MEM_ALLOCATION_TYPE_PINNED;
+  prop.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
+  prop.location.id = c->cfg.device;
+  CUmemGenericAllocationHandle h;
+  DRV_TRY(c, d.create(&h, sz, &prop, 0));
+  CUresult r = d.map(a.va + a.mapped, sz, 0, h, 0);
+  if (r != CUDA_SUCCESS) {
+    d.release(h);
+    return fail(c, VF_ERR_CUDA, "cuMemMap failed: %d", (int)r);
+  }
+  CUmemAccessDesc acc = {};
+  acc.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
+  acc.location.id = c->cfg.device;
+  acc.flags = CU_MEM_ACCESS_FLAGS_PROT_READWRITE;
+  DRV_TRY(c, d.set_access(a.va + a.mapped, sz, &acc, 1));
+  a.handles.push_back(h);
+  a.maps.push_back({a.va + a.mapped, sz});
+  a.mapped += sz;
+  return VF_OK;
+}
+
+// New region of a.next_cap objects (start at init_chunk, double).
+vf_status new_region(vf_ctx* c, Arena& a) {
+  if (a.next_cap == 0) a.next_cap = c->cfg.init_chunk_objs ? c->cfg.init_chunk_objs : 4096;
+  const uint64_t cap = a.next_cap;
+  const uint64_t bytes = cap * a.obj_bytes;
+  uint64_t start = 0;
+  void* mb = nullptr;
+  if (c->cfg.reserve_va) {
+    vf_status s = ensure_window(c, a);
+    if (s) return s;
+    s = map_upto(c, a, a.used_bytes + bytes);
+    if (s) return s;
+    start = a.va + a.used_bytes;
+    a.used_bytes += bytes;
+  } else {
+    cudaError_t e = cudaMalloc(&mb, bytes);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      return fail(c, VF_ERR_OOM, "cudaMalloc(%llu) for a region: %s", (unsigned long long)bytes,
+                  cudaGetErrorString(e));
+    }
+    start = reinterpret_cast<uint64_t>(mb);
+  }
+  vf_region r = {};
+  r.start = start;
+  r.cap_objs = cap;
+  r.used_objs = 0;
+  r.obj_bytes = a.obj_bytes;
+  r.type_id = a.type;
+  r.app = a.app;
+  c->regions.push_back(r);
+  c->region_malloc.push_back(mb);
+  a.cur = (int)c->regions.size() - 1;
+  a.next_cap = cap * 2;  // reading G3: double the previous region of this type
+  return VF_OK;
+}
+
+// Reserve `count` consecutive-in-allocation-order slots of (app,type);
+// appends their addresses to out.
+vf_status alloc_slots(vf_ctx* c, uint32_t app, uint32_t type, uint64_t count,
+                      std::vector<uint64_t>& out) {
+  const AppOps* ops = app_ops(app);
+  Arena& a = c->arenas[{app, type}];
+  if (a.obj_bytes == 0) {
+    a.app = app;
+    a.type = type;
+    a.obj_bytes = ops->obj_bytes[type];
+  }
+  out.reserve(out.size() + count);
+  while (count > 0) {
+    if (a.cur < 0 || c->regions[a.cur].used_objs == c->regions[a.cur].cap_objs) {
+      vf_status s = new_region(c, a);
+      if (s) return s;
+    }
+    vf_region& r = c->regions[a.cur];
+    const uint64_t take = std::min(count, r.cap_objs - r.used_objs);
+    for (uint64_t k = 0; k < take; ++k) out.push_back(r.start + (r.used_objs + k) * r.obj_bytes);
+    r.used_objs += take;
+    count -= take;
+  }
+  return VF_OK;
+}
+
+vf_status ensure_vptrs(vf_ctx* c, uint32_t app) {
+  AppTable& t = c->tables[app];
+  if (t.vptr_ready) return VF_OK;
+  const AppOps* ops = app_ops(app);
+  if (!t.d_vptr) CUDA_TRY(c, cudaMalloc(&t.d_vptr, sizeof(uint64_t) * ops->ntypes));
+  CUDA_TRY(c, ops->probe_vptrs(t.d_vptr, 0));
+  t.vptr.resize(ops->ntypes);
+  CUDA_TRY(c, cudaMemcpy(t.vptr.data(), t.d_vptr, sizeof(uint64_t) * ops->ntypes,
+                         cudaMemcpyDeviceToHost));
+  t.vptr_ready = true;
+  return VF_OK;
+}
+
+// Fig. 3 / P:987-991: sort the app's regions by start, merge exactly-adjacent
+// regions of the same type, upload the table for COAL.
+vf_status rebuild_table(vf_ctx* c, uint32_t app) {
+  vf_status s = ensure_vptrs(c, app);
+  if (s) return s;
+  AppTable& t = c->tables[app];
+  std::vector<const vf_region*> rs;
+  for (const vf_region& r : c->regions)
+    if (r.app == app) rs.push_back(&r);
+  std::sort(rs.begin(), rs.end(), [](const vf_region* x, const vf_region* y) { return x->start < y->start; });
+  t.rows.clear();
+  for (const vf_region* r : rs) {
+    const uint64_t e = r->start + r->cap_objs * r->obj_bytes;
+    if (!t.rows.empty() && t.rows.back().type_id == r->type_id && t.rows.back().end == r->start) {
+      t.rows.back().end = e;
+    } else {
+      vf_range row = {r->start, e, r->type_id, app, t.vptr[r->type_id]};
+      t.rows.push_back(row);
+    }
+  }
+  t.K = (uint32_t)t.rows.size();
+  t.P = 1;
+  while (t.P < t.K) t.P *= 2;
+  if (t.K > t.d_cap) {
+    cudaFree(t.d_start);
+    cudaFree(t.d_end);
+    cudaFree(t.d_type);
+    t.d_cap = std::max<uint32_t>(t.K, 64);
+    CUDA_TRY(c, cudaMalloc(&t.d_start, 8ull * t.d_cap));
+    CUDA_TRY(c, cudaMalloc(&t.d_end, 8ull * t.d_cap));
+    CUDA_TRY(c, cudaMalloc(&t.d_type, 4ull * t.d_cap));
+  }
+  if (t.K) {
+    std::vector<uint64_t> hs(t.K), he(t.K);
+    std::vector<uint32_t> ht(t.K);
+    for (uint32_t j = 0; j < t.K; ++j) {
+      hs[j] = t.rows[j].start;
+      he[j] = t.rows[j].end;
+      ht[j] = t.rows[j].type_id;
+    }
+    CUDA_TRY(c, cudaMemcpy(t.d_start, hs.data(), 8ull * t.K, cudaMemcpyHostToDevice));
+    CUDA_TRY(c, cudaMemcpy(t.d_end, he.data(), 8ull * t.K, cudaMemcpyHostToDevice));
+    CUDA_TRY(c, cudaMemcpy(t.d_type, ht.data(), 4ull * t.K, cudaMemcpyHostToDevice));
+  }
+  c->all_rows.clear();
+  for (uint32_t a = 0; a < VF_APP_COUNT; ++a)
+    c->all_rows.insert(c->all_rows.end(), c->tables[a].rows.begin(), c->tables[a].rows.end());
+  std::sort(c->all_rows.begin(), c->all_rows.end(),
+            [](const vf_range& x, const vf_range& y) { return x.start < y.start; });
+  return VF_OK;
+}
+
+DevTable dev_table(vf_ctx* c, uint32_t app) {
+  AppTable& t = c->tables[app];
+  DevTable d;
+  d.start = t.d_start;
+  d.end = t.d_end;
+  d.type = t.d_type;
+  d.K = t.K;
+  d.P = t.P;
+  d.vptr = t.d_vptr;
+  d.ntypes = app_ops(app)->ntypes;
+  d.active_types = 0;
+  for (uint64_t k : c->type_count[app]) d.active_types += (k != 0);
+  return d;
+}
+
+vf_status check_app(vf_ctx* c, uint32_t app) {
+  if (!c) return VF_ERR_INVALID;
+  if (!app_ops(app)) return fail(c, VF_ERR_INVALID, "unknown app %u", app);
+  return VF_OK;
+}
+
+const uint64_t kTagMask = ~((1ull << VF_VA_BITS) - 1);
+
+vf_status tag_check(vf_ctx* c, uint64_t addr) {
+  if (addr & kTagMask)
+    return fail(c, VF_ERR_TAG_BITS, "address 0x%llx uses bits 63:%u (TypePointer needs them 0)",
+                (unsigned long long)addr, VF_VA_BITS);
+  return VF_OK;
+}
+
+inline uint64_t tag_ptr(uint64_t addr, uint32_t type) {
+  return addr | ((uint64_t)(type + 1) << VF_VA_BITS);
+}
+
+}  // namespace
+
+extern "C" {
+
+void vf_config_default(vf_config* cfg) {
+  if (!cfg) return;
+  cfg->device = 0;
+  cfg->init_chunk_objs = 4096;
+  cfg->reserve_va = 1;
+  cfg->va_window_bytes = 64ull << 30;
+  cfg->cuda_heap_bytes = 8ull << 30;
+}
+
+const char* vf_status_str(vf_status s) {
+  switch (s) {
+    case VF_OK: return "VF_OK";
+    case VF_ERR_INVALID: return "VF_ERR_INVALID";
+    case VF_ERR_OOM: return "VF_ERR_OOM";
+    case VF_ERR_CUDA: return "VF_ERR_CUDA";
+    case VF_ERR_TAG_BITS: return "VF_ERR_TAG_BITS";
+    case VF_ERR_TOO_MANY_TYPES: return "VF_ERR_TOO_MANY_TYPES";
+    case VF_ERR_TABLE_FULL: return "VF_ERR_TABLE_FULL";
+    case VF_ERR_UNSUPPORTED: return "VF_ERR_UNSUPPORTED";
+  }
+  return "VF_ERR_?";
+}
+
+const char* vf_last_error(const vf_ctx* c) { return c ? c->err.c_str() : "null ctx"; }
+
+uint64_t vf_launch_count(void) { return g_launches.load(); }
+
+vf_status vf_set_tuning(const char* key, int value) {
+  if (!key) return VF_ERR_INVALID;
+  if (!strcmp(key, "unroll")) {
+    if (value != -1 && value != 1 && value != 2 && value != 4) return VF_ERR_INVALID;
+    tuning().unroll = value;
+  } else if (!strcmp(key, "prefetch")) {
+    tuning().prefetch = value;
+  } else {
+    return VF_ERR_INVALID;
+  }
+  return VF_OK;
+}
+
+vf_status vf_app_info(uint32_t app, uint32_t* ntypes, uint32_t* obj_bytes, uint32_t* nmethods) {
+  const AppOps* ops = app_ops(app);
+  if (!ops) return VF_ERR_INVALID;
+  if (ntypes) *ntypes = ops->ntypes;
+  if (nmethods) *nmethods = ops->nmethods;
+  if (obj_bytes)
+    for (uint32_t k = 0; k < ops->ntypes; ++k) obj_bytes[k] = ops->obj_bytes[k];
+  return VF_OK;
+}
+
+vf_status vf_create(const vf_config* cfg, vf_ctx** out) {
+  if (!out) return VF_ERR_INVALID;
+  *out = nullptr;
+  vf_ctx* c = new vf_ctx();
+  if (cfg) c->cfg = *cfg;
+  else vf_config_default(&c->cfg);
+  if (c->cfg.init_chunk_objs == 0) c->cfg.init_chunk_objs = 4096;
+  if (c->cfg.va_window_bytes == 0) c->cfg.va_window_bytes = 64ull << 30;
+  int ndev = 0;
+  cudaError_t e = cudaGetDeviceCount(&ndev);
+  if (e != cudaSuccess || c->cfg.device < 0 || c->cfg.device >= ndev) {
+    cudaGetLastError();
+    delete c;
+    return e != cudaSuccess ? VF_ERR_CUDA : VF_ERR_INVALID;
+  }
+  if (cudaSetDevice(c->cfg.device) != cudaSuccess || cudaFree(0) != cudaSuccess) {
+    delete c;
+    return VF_ERR_CUDA;
+  }
+  if (c->cfg.reserve_va) {
+    Drv& d = drv();
+    if (!d.ok) {
+      delete c;
+      return VF_ERR_UNSUPPORTED;
+    }
+    CUmemAllocationProp prop = {};
+    prop.type = CU_MEM_ALLOCATION_TYPE_PINNED;
+    prop.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
+    prop.location.id = c->cfg.device;
+    size_t g = 0;
+    if (d.granularity(&g, &prop, CU_MEM_ALLOC_GRANULARITY_RECOMMENDED) == CUDA_SUCCESS && g)
+      c->gran = g;
+  }
+  // Device heap for the CUDA baseline. The limit can only grow
+  // before the first device-malloc kernel of the process; failure here is
+  // reported later by vf_alloc_cuda.
+  if (c->cfg.cuda_heap_bytes) {
+    size_t cur = 0;
+    cudaDeviceGetLimit(&cur, cudaLimitMallocHeapSize);
+    if (cur < c->cfg.cuda_heap_bytes) {
+      if (cudaDeviceSetLimit(cudaLimitMallocHeapSize, c->cfg.cuda_heap_bytes) != cudaSuccess)
+        cudaGetLastError();
+    }
+  }
+  *out = c;
+  return VF_OK;
+}
+
+vf_status vf_reset(vf_ctx* c) {
+  if (!c) return VF_ERR_INVALID;
+  vf_status st = set_device(c);
+  if (st) return st;
+  CUDA_TRY(c, cudaDeviceSynchronize());
+  for (HeapBatch& h : c->heap) {
+    app_ops(h.app)->delete_cuda(h.d_ptrs, h.n, 0);
+    cudaDeviceSynchronize();
+    cudaFree(h.d_ptrs);
+  }
+  c->heap.clear();
+  for (size_t r = 0; r < c->region_malloc.size(); ++r)
+    if (c->region_malloc[r]) cudaFree(c->region_malloc[r]);
+  Drv& d = drv();
+  for (auto& kv : c->arenas) {
+    Arena& a = kv.second;
+    for (auto& m : a.maps) d.unmap(m.first, m.second);
+    for (auto h : a.handles) d.release(h);
+    a.maps.clear();
+    a.handles.clear();
+    a.mapped = 0;
+    a.used_bytes = 0;
+    a.cur = -1;
+    a.next_cap = 0;
+  }
+  c->regions.clear();
+  c->region_malloc.clear();
+  c->all_rows.clear();
+  for (uint32_t app = 0; app < VF_APP_COUNT; ++app) {
+    c->type_count[app].clear();
+    c->tables[app].rows.clear();
+    c->tables[app].K = 0;
+    c->tables[app].P = 1;
+  }
+  return VF_OK;
+}
+
+void vf_destroy(vf_ctx* c) {
+  if (!c) return;
+  vf_reset(c);
+  Drv& d = drv();
+  for (auto& kv : c->arenas)
+    if (kv.second.va) d.addr_free(kv.second.va, kv.second.va_size);
+  for (AppTable& t : c->tables) {
+    cudaFree(t.d_start);
+    cudaFree(t.d_end);
+    cudaFree(t.d_type);
+    cudaFree(t.d_vptr);
+  }
+  delete c;
+}
+
+vf_status vf_alloc_typed_batch(vf_ctx* c, uint32_t app, const uint32_t* type_ids_dev,
+                               uint64_t count, const void* ctor_args_dev, uint32_t ctor_arg_bytes,
+                               uint64_t* out_ptrs_dev, int tag, void* stream) {
+  vf_status st = check_app(c, app);
+  if (st) return st;
+  if (count == 0) return VF_OK;
+  if (!type_ids_dev || !out_ptrs_dev) return fail(c, VF_ERR_INVALID, "null device pointer");
+  if ((st = set_device(c))) return st;
+  const AppOps* ops = app_ops(app);
+  std::vector<uint32_t> types(count);
+  CUDA_TRY(c, cudaMemcpyAsync(types.data(), type_ids_dev, 4ull * count, cudaMemcpyDeviceToHost, S(stream)));
+  CUDA_TRY(c, cudaStreamSynchronize(S(stream)));
+  std::vector<uint64_t> cnt(ops->ntypes, 0);
+  for (uint64_t i = 0; i < count; ++i) {
+    if (types[i] >= ops->ntypes)
+      return fail(c, VF_ERR_INVALID, "type id %u at %llu >= ntypes %u", types[i],
+                  (unsigned long long)i, ops->ntypes);
+    ++cnt[types[i]];
+  }
+  if (tag && ops->ntypes > 127) return fail(c, VF_ERR_TOO_MANY_TYPES, "7-bit tag holds 127 types");
+  std::vector<std::vector<uint64_t>> slots(ops->ntypes);
+  for (uint32_t t = 0; t < ops->ntypes; ++t)
+    if (cnt[t] && (st = alloc_slots(c, app, t, cnt[t], slots[t]))) return st;
+  c->type_count[app].resize(ops->ntypes, 0);
+  for (uint32_t t = 0; t < ops->ntypes; ++t) c->type_count[app][t] += cnt[t];
+  std::vector<uint64_t> ptrs(count);
+  std::vector<uint64_t> rank(ops->ntypes, 0);
+  for (uint64_t i = 0; i < count; ++i) {
+    const uint32_t t = types[i];
+    const uint64_t a = slots[t][rank[t]++];
+    ptrs[i] = a;
+  }
+  for (uint32_t t = 0; t < ops->ntypes; ++t) {
+    if (!slots[t].empty()) {
+      if ((st = tag_check(c, slots[t].front()))) return st;
+      if ((st = tag_check(c, slots[t].back() + ops->obj_bytes[t] - 1))) return st;
+    }
+  }
+  if (tag)
+    for (uint64_t i = 0; i < count; ++i) ptrs[i] = tag_ptr(ptrs[i], types[i]);
+  CUDA_TRY(c, cudaMemcpyAsync(out_ptrs_dev, ptrs.data(), 8ull * count, cudaMemcpyHostToDevice, S(stream)));
+  CUDA_TRY(c, ops->construct(type_ids_dev, out_ptrs_dev, ctor_args_dev, ctor_arg_bytes, count, S(stream)));
+  CUDA_TRY(c, cudaStreamSynchronize(S(stream)));
+  return rebuild_table(c, app);
+}
+
+vf_status vf_alloc_typed(vf_ctx* c, uint32_t app, uint32_t type_id, uint64_t count,
+                         const void* ctor_args_dev, uint32_t ctor_arg_bytes, uint64_t* out_ptrs_dev,
+                         int tag, void* stream) {
+  vf_status st = check_app(c, app);
+  if (st) return st;
+  if (type_id >= app_ops(app)->ntypes) return fail(c, VF_ERR_INVALID, "type id %u", type_id);
+  if (count == 0) return VF_OK;
+  if ((st = set_device(c))) return st;
+  uint32_t* d_types = nullptr;
+  CUDA_TRY(c, cudaMallocAsync(&d_types, 4ull * count, S(stream)));
+  std::vector<uint32_t> h(count, type_id);
+  cudaError_t e = cudaMemcpyAsync(d_types, h.data(), 4ull * count, cudaMemcpyHostToDevice, S(stream));
+  if (e == cudaSuccess)
+    st = vf_alloc_typed_batch(c, app, d_types, count, ctor_args_dev, ctor_arg_bytes, out_ptrs_dev,
+                              tag, stream);
+  cudaFreeAsync(d_types, S(stream));
+  cudaStreamSynchronize(S(stream));
+  if (e != cudaSuccess) return fail(c, VF_ERR_CUDA, "%s", cudaGetErrorString(e));
+  return st;
+}
+
+vf_status vf_alloc_cuda(vf_ctx* c, uint32_t app, const uint32_t* type_ids_dev, uint64_t count,
+                        const void* ctor_args_dev, uint32_t ctor_arg_bytes, uint64_t* out_ptrs_dev,
+                        int tag, void* stream) {
+  vf_status st = check_app(c, app);
+  if (st) return st;
+  if (count == 0) return VF_OK;
+  if (!type_ids_dev || !out_ptrs_dev) return fail(c, VF_ERR_INVALID, "null device pointer");
+  if ((st = set_device(c))) return st;
+  const AppOps* ops = app_ops(app);
+  if (tag && ops->ntypes > 127) return fail(c, VF_ERR_TOO_MANY_TYPES, "7-bit tag holds 127 types");
+  CUDA_TRY(c, ops->new_cuda(type_ids_dev, ctor_args_dev, ctor_arg_bytes, count, out_ptrs_dev, S(stream)));
+  CUDA_TRY(c, cudaStreamSynchronize(S(stream)));
+  std::vector<uint64_t> ptrs(count);
+  CUDA_TRY(c, cudaMemcpy(ptrs.data(), out_ptrs_dev, 8ull * count, cudaMemcpyDeviceToHost));
+  uint64_t nulls = 0;
+  for (uint64_t p : ptrs) nulls += (p == 0);
+  // keep an untagged copy for delete
+  HeapBatch hb{app, nullptr, count};
+  CUDA_TRY(c, cudaMalloc(&hb.d_ptrs, 8ull * count));
+  CUDA_TRY(c, cudaMemcpy(hb.d_ptrs, out_ptrs_dev, 8ull * count, cudaMemcpyDeviceToDevice));
+  c->heap.push_back(hb);
+  if (nulls)
+    return fail(c, VF_ERR_OOM, "device heap exhausted: %llu of %llu `new` returned null (raise cuda_heap_bytes before the first device-malloc kernel)",
+                (unsigned long long)nulls, (unsigned long long)count);
+  for (uint64_t p : ptrs)
+    if ((st = tag_check(c, p))) return st;
+  std::vector<uint32_t> types(count);
+  CUDA_TRY(c, cudaMemcpy(types.data(), type_ids_dev, 4ull * count, cudaMemcpyDeviceToHost));
+  c->type_count[app].resize(ops->ntypes, 0);
+  for (uint32_t t : types)
+    if (t < ops->ntypes) ++c->type_count[app][t];
+  if (tag) {
+    for (uint64_t i = 0; i < count; ++i) ptrs[i] = tag_ptr(ptrs[i], types[i]);
+    CUDA_TRY(c, cudaMemcpy(out_ptrs_dev, ptrs.data(), 8ull * count, cudaMemcpyHostToDevice));
+  }
+  return ensure_vptrs(c, app);
+}
+
+vf_status vf_range_table(const vf_ctx* c, uint32_t app, const vf_range** out, uint32_t* n) {
+  if (!c || !out || !n) return VF_ERR_INVALID;
+  if (app == 0xFFFFFFFFu) {
+    *out = c->all_rows.data();
+    *n = (uint32_t)c->all_rows.size();
+    return VF_OK;
+  }
+  if (app >= VF_APP_COUNT) return VF_ERR_INVALID;
+  *out = c->tables[app].rows.data();
+  *n = (uint32_t)c->tables[app].rows.size();
+  return VF_OK;
+}
+
+vf_status vf_regions(const vf_ctx* c, const vf_region** out, uint32_t* n) {
+  if (!c || !out || !n) return VF_ERR_INVALID;
+  *out = c->regions.data();
+  *n = (uint32_t)c->regions.size();
+  return VF_OK;
+}
+
+vf_status vf_type_vptrs(vf_ctx* c, uint32_t app, uint64_t* vptrs_out) {
+  vf_status st = check_app(c, app);
+  if (st) return st;
+  if ((st = set_device(c)) || (st = ensure_vptrs(c, app))) return st;
+  if (vptrs_out)
+    std::copy(c->tables[app].vptr.begin(), c->tables[app].vptr.end(), vptrs_out);
+  return VF_OK;
+}
+
+vf_status vf_resolve(vf_ctx* c, uint32_t app, vf_variant v, const uint64_t* ptrs_dev, uint64_t n,
+                     uint32_t* types_out_dev, void* stream) {
+  vf_status st = check_app(c, app);
+  if (st) return st;
+  if ((unsigned)v > VF_TYPEPTR) return fail(c, VF_ERR_INVALID, "variant %d", (int)v);
+  if ((st = set_device(c)) || (st = ensure_vptrs(c, app))) return st;
+  if (v == VF_COAL && c->tables[app].K > VF_MAX_RANGES)
+    return fail(c, VF_ERR_TABLE_FULL, "K = %u > %u", c->tables[app].K, VF_MAX_RANGES);
+  CUDA_TRY(c, app_ops(app)->resolve((int)v, ptrs_dev, n, types_out_dev, dev_table(c, app), S(stream)));
+  return VF_OK;
+}
+
+vf_status vf_verify_types(vf_ctx* c, uint32_t app, vf_variant v, const uint64_t* ptrs_dev,
+                          uint64_t n, unsigned long long* mism_dev, void* stream) {
+  vf_status st = check_app(c, app);
+  if (st) return st;
+  if ((unsigned)v > VF_TYPEPTR) return fail(c, VF_ERR_INVALID, "variant %d", (int)v);
+  if ((st = set_device(c)) || (st = ensure_vptrs(c, app))) return st;
+  if (v == VF_COAL && c->tables[app].K > VF_MAX_RANGES)
+    return fail(c, VF_ERR_TABLE_FULL, "K = %u > %u", c->tables[app].K, VF_MAX_RANGES);
+  CUDA_TRY(c, app_ops(app)->verify((int)v, ptrs_dev, n, mism_dev, dev_table(c, app), S(stream)));
+  return VF_OK;
+}
+
+vf_status vf_dispatch(vf_ctx* c, vf_variant v, uint32_t app, uint32_t method,
+                      const uint64_t* objs_dev, uint64_t n, const void* args, size_t args_bytes,
+                      void* stream) {
+  vf_status st = check_app(c, app);
+  if (st) return st;
+  const AppOps* ops = app_ops(app);
+  if ((unsigned)v > VF_TYPEPTR) return fail(c, VF_ERR_INVALID, "variant %d", (int)v);
+  if (method >= ops->nmethods) return fail(c, VF_ERR_INVALID, "method %u of app %s", method, ops->name);
+  if (args_bytes > VF_MAX_ARGS_BYTES || (args_bytes && !args))
+    return fail(c, VF_ERR_INVALID, "args_bytes %zu", args_bytes);
+  if (args_bytes < ops->method_args_bytes[method])
+    return fail(c, VF_ERR_INVALID, "method %u needs %u argument bytes, got %zu", method,
+                ops->method_args_bytes[method], args_bytes);
+  if (n && !objs_dev) return fail(c, VF_ERR_INVALID, "null objs");
+  if (v == VF_COAL && c->tables[app].K > VF_MAX_RANGES)
+    return fail(c, VF_ERR_TABLE_FULL, "K = %u > %u", c->tables[app].K, VF_MAX_RANGES);
+  ArgBlob blob;
+  memset(&blob, 0, sizeof blob);
+  if (args_bytes) memcpy(blob.b, args, args_bytes);
+  CUDA_TRY(c, ops->dispatch((int)v, method, objs_dev, n, blob, dev_table(c, app), S(stream)));
+  return VF_OK;
+}
+
+vf_status vf_dispatch_cuda(vf_ctx* c, uint32_t app, uint32_t m, const uint64_t* o, uint64_t n,
+                           const void* a, size_t ab, void* s) {
+  return vf_dispatch(c, VF_CUDA, app, m, o, n, a, ab, s);
+}
+vf_status vf_dispatch_sharedoa(vf_ctx* c, uint32_t app, uint32_t m, const uint64_t* o, uint64_t n,
+                               const void* a, size_t ab, void* s) {
+  return vf_dispatch(c, VF_SHAREDOA, app, m, o, n, a, ab, s);
+}
+vf_status vf_dispatch_coal(vf_ctx* c, uint32_t app, uint32_t m, const uint64_t* o, uint64_t n,
+                           const void* a, size_t ab, void* s) {
+  return vf_dispatch(c, VF_COAL, app, m, o, n, a, ab, s);
+}
+vf_status vf_dispatch_typeptr(vf_ctx* c, uint32_t app, uint32_t m, const uint64_t* o, uint64_t n,
+                              const void* a, size_t ab, void* s) {
+  return vf_dispatch(c, VF_TYPEPTR, app, m, o, n, a, ab, s);
+}
+
+}  // extern "C"

@@ -1,0 +1,73 @@
+// vf_internal.h — internal interface between the host core (core.cu) and the
+// per-app device modules (app_*.cu). Not part of the public ABI (include/vf.h).
+//
+// GPUs cannot load code dynamically: every virtual function a kernel may call
+// must be compiled into that kernel's module, and a vTable* is only
+// meaningful inside the module whose kernel constructed the object. So each app
+// is ONE translation unit holding its class hierarchy, its construction kernels
+// and its dispatch kernels, and exports an AppOps table to the core.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "../../include/vf.h"
+
+namespace vf {
+
+// Method argument blob, copied by value into kernel parameters.
+struct __align__(16) ArgBlob {
+  unsigned char b[VF_MAX_ARGS_BYTES];
+};
+
+// Device view of one app's virtual range table (sorted, merged) and vTables.
+struct DevTable {
+  const uint64_t* start;  // K entries, sorted
+  const uint64_t* end;    // K entries
+  const uint32_t* type;   // K entries
+  uint32_t K;
+  uint32_t P;             // K rounded up to a power of two (>= 1); smem table size
+  const uint64_t* vptr;   // ntypes entries: device vTable* per concrete type
+  uint32_t ntypes;
+  uint32_t active_types;  // concrete types with live objects (launch heuristics)
+};
+
+struct AppOps {
+  const char* name;
+  uint32_t ntypes;
+  const uint32_t* obj_bytes;  // per type, sizeof(class)
+  uint32_t nmethods;
+  const uint32_t* method_args_bytes;  // per method: sizeof(args struct)
+  // vTable* of each type -> out_dev[ntypes] (placement-new into scratch).
+  cudaError_t (*probe_vptrs)(uint64_t* out_dev, cudaStream_t s);
+  // placement-new object i of class types[i] at strip(ptrs[i]).
+  cudaError_t (*construct)(const uint32_t* types_dev, const uint64_t* ptrs_dev,
+                           const void* ctor_args_dev, uint32_t ctor_arg_bytes, uint64_t n,
+                           cudaStream_t s);
+  // device-heap new (CUDA baseline); out_ptrs[i] = new T(types[i]) or 0.
+  cudaError_t (*new_cuda)(const uint32_t* types_dev, const void* ctor_args_dev,
+                          uint32_t ctor_arg_bytes, uint64_t n, uint64_t* out_ptrs_dev,
+                          cudaStream_t s);
+  // delete of device-heap objects (untagged pointers).
+  cudaError_t (*delete_cuda)(const uint64_t* ptrs_dev, uint64_t n, cudaStream_t s);
+  cudaError_t (*dispatch)(int variant, uint32_t method, const uint64_t* objs_dev, uint64_t n,
+                          const ArgBlob& args, const DevTable& tbl, cudaStream_t s);
+  cudaError_t (*resolve)(int variant, const uint64_t* ptrs_dev, uint64_t n, uint32_t* out_dev,
+                         const DevTable& tbl, cudaStream_t s);
+  cudaError_t (*verify)(int variant, const uint64_t* ptrs_dev, uint64_t n,
+                        unsigned long long* mism_dev, const DevTable& tbl, cudaStream_t s);
+};
+
+const AppOps* app_micro();
+const AppOps* app_gol();
+
+// Benchmark / ablation knobs set through vf_set_tuning (-1 = app default).
+struct Tuning {
+  int unroll = -1;    // objects per thread in the grouped kernels (1, 2, 4)
+  int prefetch = -1;  // 1: prefetch object lines to L1 before the type groups
+};
+Tuning& tuning();
+
+// launch accounting (bench: gpu_launches)
+void note_launch(uint64_t k = 1);
+
+}  // namespace vf

@@ -1,0 +1,312 @@
+"""Thin ctypes binding of libvf.so (include/vf.h) — argument marshalling only.
+
+Every step of the path runs in libvf's CUDA kernels; torch supplies device
+memory (tensors' data_ptr()) and streams. There is no CPU fallback: if
+libvf.so is missing or no CUDA device is present, constructing a Ctx raises.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass
+
+import numpy as np
+
+PKG = os.path.dirname(os.path.abspath(__file__))
+SO = os.path.join(PKG, "libvf.so")
+
+# enums mirrored from include/vf.h
+VF_OK = 0
+CUDA, SHAREDOA, COAL, TYPEPTR = 0, 1, 2, 3
+VARIANTS = {"cuda": CUDA, "sharedoa": SHAREDOA, "coal": COAL, "typeptr": TYPEPTR}
+APP_MICRO, APP_GOL = 0, 1
+MICRO_APPLY, MICRO_GET = 0, 1
+GOL_NEXT, GOL_GET = 0, 1
+NOT_FOUND = 0xFFFFFFFF
+VA_BITS = 57
+MAX_RANGES = 4096
+
+STATUS = {0: "VF_OK", 1: "VF_ERR_INVALID", 2: "VF_ERR_OOM", 3: "VF_ERR_CUDA", 4: "VF_ERR_TAG_BITS",
+          5: "VF_ERR_TOO_MANY_TYPES", 6: "VF_ERR_TABLE_FULL", 7: "VF_ERR_UNSUPPORTED"}
+
+# exported symbols (checked by tests/test_abi.py against include/vf.h)
+SYMBOLS = [
+    "vf_config_default", "vf_create", "vf_destroy", "vf_status_str", "vf_last_error", "vf_app_info",
+    "vf_alloc_typed", "vf_alloc_typed_batch", "vf_alloc_cuda", "vf_reset", "vf_range_table",
+    "vf_regions", "vf_type_vptrs", "vf_resolve", "vf_verify_types", "vf_dispatch_cuda",
+    "vf_dispatch_sharedoa", "vf_dispatch_coal", "vf_dispatch_typeptr", "vf_dispatch",
+    "vf_gol_neighbors", "vf_gol_swap", "vf_checksum_i32", "vf_launch_count", "vf_set_tuning",
+]
+
+
+class VFError(RuntimeError):
+    def __init__(self, status, msg=""):
+        super().__init__(f"{STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+class vf_config(ctypes.Structure):
+    _fields_ = [("device", ctypes.c_int), ("init_chunk_objs", ctypes.c_uint64),
+                ("reserve_va", ctypes.c_int), ("va_window_bytes", ctypes.c_uint64),
+                ("cuda_heap_bytes", ctypes.c_uint64)]
+
+
+class vf_range(ctypes.Structure):
+    _fields_ = [("start", ctypes.c_uint64), ("end", ctypes.c_uint64), ("type_id", ctypes.c_uint32),
+                ("app", ctypes.c_uint32), ("vptr", ctypes.c_uint64)]
+
+
+class vf_region(ctypes.Structure):
+    _fields_ = [("start", ctypes.c_uint64), ("cap_objs", ctypes.c_uint64),
+                ("used_objs", ctypes.c_uint64), ("obj_bytes", ctypes.c_uint32),
+                ("type_id", ctypes.c_uint32), ("app", ctypes.c_uint32), ("pad", ctypes.c_uint32)]
+
+
+class micro_get_args(ctypes.Structure):
+    _fields_ = [("out_dev", ctypes.c_void_p)]
+
+
+class gol_next_args(ctypes.Structure):
+    _fields_ = [("nbr_dev", ctypes.c_void_p), ("state_out_dev", ctypes.c_void_p)]
+
+
+class gol_get_args(ctypes.Structure):
+    _fields_ = [("counter_out_dev", ctypes.c_void_p), ("type_out_dev", ctypes.c_void_p)]
+
+
+_lib = None
+
+
+def lib(required: bool = True):
+    """Load libvf.so (fails loudly when it is missing: there is no fallback)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(SO):
+        raise FileNotFoundError(f"{SO} not built: run __graft_entry__.build()")
+    L = ctypes.CDLL(SO)
+    P, U32, U64, I = ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_int
+    sig = {
+        "vf_config_default": (None, [ctypes.POINTER(vf_config)]),
+        "vf_create": (I, [ctypes.POINTER(vf_config), ctypes.POINTER(P)]),
+        "vf_destroy": (None, [P]),
+        "vf_status_str": (ctypes.c_char_p, [I]),
+        "vf_last_error": (ctypes.c_char_p, [P]),
+        "vf_app_info": (I, [U32, ctypes.POINTER(U32), ctypes.POINTER(U32), ctypes.POINTER(U32)]),
+        "vf_alloc_typed": (I, [P, U32, U32, U64, P, U32, P, I, P]),
+        "vf_alloc_typed_batch": (I, [P, U32, P, U64, P, U32, P, I, P]),
+        "vf_alloc_cuda": (I, [P, U32, P, U64, P, U32, P, I, P]),
+        "vf_reset": (I, [P]),
+        "vf_range_table": (I, [P, U32, ctypes.POINTER(ctypes.POINTER(vf_range)), ctypes.POINTER(U32)]),
+        "vf_regions": (I, [P, ctypes.POINTER(ctypes.POINTER(vf_region)), ctypes.POINTER(U32)]),
+        "vf_type_vptrs": (I, [P, U32, P]),
+        "vf_resolve": (I, [P, U32, I, P, U64, P, P]),
+        "vf_verify_types": (I, [P, U32, I, P, U64, P, P]),
+        "vf_dispatch": (I, [P, I, U32, U32, P, U64, P, ctypes.c_size_t, P]),
+        "vf_dispatch_cuda": (I, [P, U32, U32, P, U64, P, ctypes.c_size_t, P]),
+        "vf_dispatch_sharedoa": (I, [P, U32, U32, P, U64, P, ctypes.c_size_t, P]),
+        "vf_dispatch_coal": (I, [P, U32, U32, P, U64, P, ctypes.c_size_t, P]),
+        "vf_dispatch_typeptr": (I, [P, U32, U32, P, U64, P, ctypes.c_size_t, P]),
+        "vf_gol_neighbors": (I, [U32, U32, I, P, P, P]),
+        "vf_gol_swap": (I, [P, U64, P, P, P, P, P, P]),
+        "vf_checksum_i32": (I, [P, U64, P, P]),
+        "vf_launch_count": (U64, []),
+        "vf_set_tuning": (I, [ctypes.c_char_p, I]),
+    }
+    for name, (res, args) in sig.items():
+        f = getattr(L, name)
+        f.restype = res
+        f.argtypes = args
+    _lib = L
+    return L
+
+
+def app_info(app: int):
+    L = lib()
+    nt, nm = ctypes.c_uint32(), ctypes.c_uint32()
+    sizes = (ctypes.c_uint32 * 128)()
+    st = L.vf_app_info(app, ctypes.byref(nt), sizes, ctypes.byref(nm))
+    if st:
+        raise VFError(st, f"app {app}")
+    return int(nt.value), [int(sizes[k]) for k in range(nt.value)], int(nm.value)
+
+
+def set_tuning(key: str, value: int):
+    st = lib().vf_set_tuning(key.encode(), int(value))
+    if st:
+        raise VFError(st, f"tuning {key}={value}")
+
+
+def launch_count() -> int:
+    return int(lib().vf_launch_count())
+
+
+def _ptr(t) -> int | None:
+    if t is None:
+        return None
+    return int(t.data_ptr())
+
+
+def _stream(stream) -> int | None:
+    import torch
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return int(s.cuda_stream) if hasattr(s, "cuda_stream") else int(s)
+
+
+def _args(a) -> tuple:
+    if a is None:
+        return None, 0
+    return ctypes.cast(ctypes.pointer(a), ctypes.c_void_p), ctypes.sizeof(a)
+
+
+@dataclass
+class Range:
+    start: int
+    end: int
+    type_id: int
+    app: int
+    vptr: int
+
+
+class Ctx:
+    """One vf_ctx (per process and device). Owns every object it allocates."""
+
+    def __init__(self, device: int = 0, init_chunk_objs: int = 4096, reserve_va: bool = True,
+                 va_window_bytes: int = 64 << 30, cuda_heap_bytes: int = 8 << 30):
+        import torch
+        if not torch.cuda.is_available():
+            raise RuntimeError("libvf needs a CUDA device (no CPU fallback)")
+        L = lib()
+        cfg = vf_config()
+        L.vf_config_default(ctypes.byref(cfg))
+        cfg.device, cfg.init_chunk_objs, cfg.reserve_va = device, init_chunk_objs, int(reserve_va)
+        cfg.va_window_bytes, cfg.cuda_heap_bytes = va_window_bytes, cuda_heap_bytes
+        h = ctypes.c_void_p()
+        st = L.vf_create(ctypes.byref(cfg), ctypes.byref(h))
+        if st:
+            raise VFError(st, "vf_create")
+        self.h = h
+        self.device = device
+        self.L = L
+
+    def _check(self, st, what=""):
+        if st:
+            raise VFError(st, f"{what}: {self.L.vf_last_error(self.h).decode(errors='replace')}")
+
+    def close(self):
+        if getattr(self, "h", None):
+            self.L.vf_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    # ---- allocation ---------------------------------------------------------
+    def alloc_typed_batch(self, app, types, ctor_args=None, tag=False, stream=None):
+        """types: int32/uint32 CUDA tensor [n]; ctor_args: CUDA tensor [n, ...] (contiguous).
+        Returns an int64 CUDA tensor of object pointers (tagged if tag)."""
+        import torch
+        n = types.numel()
+        out = torch.empty(n, dtype=torch.int64, device=types.device)
+        ab = 0 if ctor_args is None else ctor_args.element_size() * (ctor_args.numel() // max(n, 1))
+        self._check(self.L.vf_alloc_typed_batch(self.h, app, _ptr(types), n, _ptr(ctor_args), ab,
+                                                _ptr(out), int(tag), _stream(stream)), "alloc_typed_batch")
+        return out
+
+    def alloc_typed(self, app, type_id, count, ctor_args=None, tag=False, stream=None):
+        import torch
+        out = torch.empty(count, dtype=torch.int64, device=f"cuda:{self.device}")
+        ab = 0 if ctor_args is None else ctor_args.element_size() * (ctor_args.numel() // max(count, 1))
+        self._check(self.L.vf_alloc_typed(self.h, app, type_id, count, _ptr(ctor_args), ab, _ptr(out),
+                                          int(tag), _stream(stream)), "alloc_typed")
+        return out
+
+    def alloc_cuda(self, app, types, ctor_args=None, tag=False, stream=None):
+        import torch
+        n = types.numel()
+        out = torch.empty(n, dtype=torch.int64, device=types.device)
+        ab = 0 if ctor_args is None else ctor_args.element_size() * (ctor_args.numel() // max(n, 1))
+        self._check(self.L.vf_alloc_cuda(self.h, app, _ptr(types), n, _ptr(ctor_args), ab, _ptr(out),
+                                         int(tag), _stream(stream)), "alloc_cuda")
+        return out
+
+    def reset(self):
+        self._check(self.L.vf_reset(self.h), "reset")
+
+    # ---- tables -------------------------------------------------------------
+    def range_table(self, app=0xFFFFFFFF):
+        p = ctypes.POINTER(vf_range)()
+        n = ctypes.c_uint32()
+        self._check(self.L.vf_range_table(self.h, app, ctypes.byref(p), ctypes.byref(n)), "range_table")
+        return [Range(p[k].start, p[k].end, p[k].type_id, p[k].app, p[k].vptr) for k in range(n.value)]
+
+    def regions(self):
+        p = ctypes.POINTER(vf_region)()
+        n = ctypes.c_uint32()
+        self._check(self.L.vf_regions(self.h, ctypes.byref(p), ctypes.byref(n)), "regions")
+        return [dict(start=p[k].start, cap_objs=p[k].cap_objs, used_objs=p[k].used_objs,
+                     obj_bytes=p[k].obj_bytes, type_id=p[k].type_id, app=p[k].app)
+                for k in range(n.value)]
+
+    def type_vptrs(self, app):
+        nt, _, _ = app_info(app)
+        buf = (ctypes.c_uint64 * nt)()
+        self._check(self.L.vf_type_vptrs(self.h, app, buf), "type_vptrs")
+        return [int(x) for x in buf]
+
+    # ---- resolve / verify / dispatch -----------------------------------------
+    def resolve(self, app, variant, ptrs, stream=None):
+        import torch
+        out = torch.empty(ptrs.numel(), dtype=torch.int32, device=ptrs.device)
+        self._check(self.L.vf_resolve(self.h, app, variant, _ptr(ptrs), ptrs.numel(), _ptr(out),
+                                      _stream(stream)), "resolve")
+        return out
+
+    def verify(self, app, variant, ptrs, stream=None) -> int:
+        import torch
+        m = torch.zeros(1, dtype=torch.int64, device=ptrs.device)
+        self._check(self.L.vf_verify_types(self.h, app, variant, _ptr(ptrs), ptrs.numel(), _ptr(m),
+                                           _stream(stream)), "verify_types")
+        return int(m.item())
+
+    def dispatch(self, variant, app, method, objs, args=None, n=None, stream=None):
+        a, ab = _args(args)
+        n = objs.numel() if n is None else n
+        self._check(self.L.vf_dispatch(self.h, variant, app, method, _ptr(objs), n, a, ab,
+                                       _stream(stream)), "dispatch")
+
+    def dispatch_raw(self, variant, app, method, objs_ptr: int, n: int, args=None, stream=None):
+        """Same as dispatch() with a raw device pointer (hot loops avoid tensor overhead)."""
+        a, ab = _args(args)
+        return self.L.vf_dispatch(self.h, variant, app, method, objs_ptr, n, a, ab, stream)
+
+
+def gol_neighbors(W, H, state, nbr, torus=False, stream=None):
+    st = lib().vf_gol_neighbors(W, H, int(torus), _ptr(state), _ptr(nbr), _stream(stream))
+    if st:
+        raise VFError(st, "gol_neighbors")
+
+
+def gol_swap(ctx: Ctx, prev, nxt, grid, alive, dead, stream=None):
+    st = lib().vf_gol_swap(ctx.h, grid.numel(), _ptr(prev), _ptr(nxt), _ptr(grid), _ptr(alive),
+                           _ptr(dead), _stream(stream))
+    if st:
+        raise VFError(st, "gol_swap")
+
+
+def checksum_i32(vals, out, stream=None):
+    st = lib().vf_checksum_i32(_ptr(vals), vals.numel(), _ptr(out), _stream(stream))
+    if st:
+        raise VFError(st, "checksum_i32")
+
+
+def strip(p: int) -> int:
+    return p & ((1 << VA_BITS) - 1)
+
+
+def as_u64(t) -> np.ndarray:
+    """int64 torch tensor of pointers -> numpy uint64 (bit pattern)."""
+    return t.cpu().numpy().view(np.uint64)
