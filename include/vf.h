@@ -215,9 +215,13 @@ vf_status vf_gol_swap(vf_ctx* ctx, uint64_t ncells, const uint8_t* state_prev_de
 /* sum over i of vals_dev[i] (int32, widened) into *out_dev (i64, device). */
 vf_status vf_checksum_i32(const int32_t* vals_dev, uint64_t n, long long* out_dev, void* stream);
 /* Benchmark / ablation knobs of the COAL / TYPEPTR kernels (process-wide):
- * "unroll" = objects per thread (1, 2, 4; -1 = app default), "prefetch" =
- * 1/0 to issue (or not) an L1 prefetch of every object line before the type
- * groups run (-1 = default on). VF_ERR_INVALID for unknown keys / values. */
+ * "unroll" = objects per thread (1, 2, 4; -1 = app default); "prefetch" =
+ * object-line warm-up before the type groups (0 none, 1 prefetch.global.L1,
+ * 2 L1-allocating load; -1 = app default); "regroup" = 1 (default) sorts
+ * each CTA tile by type in shared memory before the calls, 0 groups within
+ * warps only; "pipeline" = 1 streams the pointer array through a TMA /
+ * mbarrier ring in shared memory (regroup 0 only), 0 (default) uses plain
+ * per-thread loads. VF_ERR_INVALID for unknown keys / values. */
 vf_status vf_set_tuning(const char* key, int value);
 /* Number of libvf kernel launches issued since load (for bench accounting). */
 uint64_t vf_launch_count(void);

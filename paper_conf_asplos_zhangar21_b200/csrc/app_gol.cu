@@ -59,6 +59,7 @@ struct App {
   static constexpr int kTypes = 2;  // 0 = Dead, 1 = Alive
   static constexpr int kMethods = 2;
   static constexpr int kUnroll = 1;
+  static constexpr int kUnrollSorted = 2;
   static constexpr int kPrefetch = 0;
   using Base = Cell;
   template <int K>

@@ -29,6 +29,7 @@ struct App {
   static constexpr int kTypes = 32;
   static constexpr int kMethods = 2;
   static constexpr int kUnroll = 2;
+  static constexpr int kUnrollSorted = 2;
   static constexpr int kPrefetch = 2;
   using Base = MObj;
   template <int K>

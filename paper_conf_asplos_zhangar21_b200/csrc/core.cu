@@ -400,7 +400,14 @@ vf_status vf_set_tuning(const char* key, int value) {
     if (value != -1 && value != 1 && value != 2 && value != 4) return VF_ERR_INVALID;
     tuning().unroll = value;
   } else if (!strcmp(key, "prefetch")) {
+    if (value < -1 || value > 2) return VF_ERR_INVALID;
     tuning().prefetch = value;
+  } else if (!strcmp(key, "regroup")) {
+    if (value < 0 || value > 1) return VF_ERR_INVALID;
+    tuning().regroup = value;
+  } else if (!strcmp(key, "pipeline")) {
+    if (value < 0 || value > 1) return VF_ERR_INVALID;
+    tuning().pipeline = value;
   } else {
     return VF_ERR_INVALID;
   }

@@ -43,6 +43,8 @@ __device__ __forceinline__ uint64_t ldg_u64(const uint64_t* p) {
   return v;
 }
 
+__host__ __device__ constexpr size_t table_smem_dev(uint32_t P) { return (size_t)P * (8 + 8 + 4); }
+
 __device__ __forceinline__ void prefetch_l1(uint64_t a) {
   asm volatile("prefetch.global.L1 [%0];" ::"l"(a));
 }
@@ -59,7 +61,7 @@ struct ResolveTP {
   static constexpr bool kNeedsTable = false;
   __device__ static void stage(unsigned char*, const DevTable&) {}
   __device__ __forceinline__ static uint32_t resolve(const unsigned char*, uint32_t,
-                                                     uint64_t p, uint64_t& a) {
+                                                     uint64_t p, uint64_t& a, uint32_t&) {
     a = strip(p);
     const uint32_t tag = (uint32_t)(p >> 32) >> (VF_VA_BITS - 32);
     return tag - 1u;  // tag 0 (untagged) -> 0xFFFFFFFF = not found -> fallback
@@ -85,16 +87,22 @@ struct ResolveCOAL {
     }
     __syncthreads();
   }
+  // `hint` = the lane's previous range: consecutive objects of a lane usually
+  // fall in the same range, so the search runs only on a miss.
   __device__ __forceinline__ static uint32_t resolve(const unsigned char* smem, uint32_t P,
-                                                     uint64_t p, uint64_t& a) {
+                                                     uint64_t p, uint64_t& a, uint32_t& hint) {
     const uint64_t* s_start = reinterpret_cast<const uint64_t*>(smem);
     const uint64_t* s_end = s_start + P;
     const uint32_t* s_type = reinterpret_cast<const uint32_t*>(s_end + P);
     a = p;
-    uint32_t j = 0;
-    for (uint32_t step = P >> 1; step > 0; step >>= 1) {
-      const uint32_t c = j + step;
-      j = (s_start[c] <= p) ? c : j;
+    uint32_t j = hint;
+    if (!((s_start[j] <= p) & (p < s_end[j]))) {
+      j = 0;
+      for (uint32_t step = P >> 1; step > 0; step >>= 1) {
+        const uint32_t c = j + step;
+        j = (s_start[c] <= p) ? c : j;
+      }
+      hint = j;
     }
     const bool hit = (s_start[j] <= p) & (p < s_end[j]);
     return hit ? s_type[j] : kNF;
@@ -129,9 +137,29 @@ __device__ __forceinline__ void select_body(uint32_t k, uint32_t t, uint64_t a, 
   }
 }
 
+// Fallback ("use COAL or the traditional CUDA vFunc lookup as a
+// backup"): a non-null pointer the resolver could not place (COAL miss, tag 0)
+// is typed by its embedded vTable*, matched against the app's per-type vTable*
+// table, and then joins the same grouped direct call. No CALL instruction is
+// emitted anywhere in the grouped kernels, so they are not subject to the
+// call ABI (which caps a calling kernel at 32 registers on sm_100a).
+template <class App>
+__device__ __forceinline__ uint32_t type_from_vptr(uint64_t a, const DevTable& tbl) {
+  const uint64_t vp = *reinterpret_cast<const uint64_t*>(a);
+  uint32_t t = kNF;
+#pragma unroll 1
+  for (uint32_t k = 0; k < (uint32_t)App::kTypes; ++k)
+    if (tbl.vptr[k] == vp) t = k;
+  return t;
+}
+
 template <class App, int M>
 __device__ __forceinline__ void group_call(uint32_t t, uint64_t a, uint64_t p, uint64_t i,
-                                           const ArgBlob& args) {
+                                           const ArgBlob& args, const DevTable& tbl) {
+  const bool fb = t >= (uint32_t)App::kTypes && p != 0;
+  if (__any_sync(0xffffffffu, fb)) {
+    if (fb) t = type_from_vptr<App>(a, tbl);
+  }
   const bool ok = t < (uint32_t)App::kTypes;
   uint32_t present = __reduce_or_sync(0xffffffffu, ok ? (1u << t) : 0u);
   if constexpr (App::kTypes == 1) {
@@ -142,11 +170,6 @@ __device__ __forceinline__ void group_call(uint32_t t, uint64_t a, uint64_t p, u
       present &= present - 1;
       select_body<App, M, 0, App::kTypes>(k, t, a, i, args);
     }
-  }
-  // Fallback: unresolved non-null pointer -> embedded vTable*.
-  const bool fb = !ok && p != 0;
-  if (__any_sync(0xffffffffu, fb)) {
-    if (fb) App::template vcall<M>(reinterpret_cast<typename App::Base*>(a), i, args);
   }
 }
 
@@ -173,6 +196,7 @@ __global__ void __launch_bounds__(kBlock) k_dispatch_grouped(const uint64_t* __r
   if constexpr (R::kNeedsTable) R::stage(smem, tbl);
   const uint64_t tile = (uint64_t)kBlock * U;
   uint32_t sink = 0;
+  uint32_t hint = 0;  // COAL: last range hit by this lane
   for (uint64_t base = (uint64_t)blockIdx.x * tile; base < n; base += (uint64_t)gridDim.x * tile) {
     uint64_t p[U];
 #pragma unroll
@@ -184,7 +208,7 @@ __global__ void __launch_bounds__(kBlock) k_dispatch_grouped(const uint64_t* __r
     uint32_t t[U];
 #pragma unroll
     for (int j = 0; j < U; ++j) {
-      t[j] = p[j] ? R::resolve(smem, tbl.P, p[j], a[j]) : kNF;
+      t[j] = p[j] ? R::resolve(smem, tbl.P, p[j], a[j], hint) : kNF;
       if (!p[j]) a[j] = 0;
     }
     // Issue every lane's object line before the (serialised) type groups run,
@@ -198,11 +222,313 @@ __global__ void __launch_bounds__(kBlock) k_dispatch_grouped(const uint64_t* __r
 #pragma unroll
     for (int j = 0; j < U; ++j) {
       const uint64_t idx = base + (uint64_t)j * kBlock + threadIdx.x;
-      group_call<App, M>(t[j], a[j], p[j], idx, args);
+      group_call<App, M>(t[j], a[j], p[j], idx, args, tbl);
     }
   }
   if constexpr (PF == 2) {
     // never true for a valid launch (n < 2^64-1); keeps the warm-up loads alive
+    if (sink == 0x8BADF00Du && n == ~0ull) asm volatile("st.global.u32 [%0], %1;" ::"l"(objs), "r"(sink));
+  }
+}
+
+// ---------------------------------------------------------------------------
+// TMA-pipelined grouped dispatch (default for COAL / TypePointer).
+//
+// The pointer array is a pure stream: one elected thread per CTA moves each
+// tile of kBlock*U pointers global -> shared with cp.async.bulk (TMA, 1-D)
+// into an S-stage ring completed on mbarriers, so pointer latency never sits
+// on a warp's critical path. The warps run one tile ahead on the objects:
+// while tile k's type groups execute, tile k+1's pointers are already resolved
+// and its object lines are in flight (warm loads), i.e. one DRAM round trip of
+// objects overlaps every group walk.
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return (uint32_t)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  uint32_t done;
+  do {
+    asm volatile(
+        "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n"
+        " selp.u32 %0, 1, 0, p;\n}\n"
+        : "=r"(done)
+        : "r"(smem_u32(bar)), "r"(parity)
+        : "memory");
+  } while (!done);
+}
+__device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+
+__host__ __device__ constexpr size_t align16(size_t x) { return (x + 15) & ~(size_t)15; }
+
+template <int U, int S>
+struct PipeSmem {
+  static constexpr int kWarps = kBlock / 32;
+  static constexpr int kTile = 32 * U;  // objects per warp tile
+  static constexpr size_t kRing = (size_t)kWarps * S * kTile * sizeof(uint64_t);
+  static constexpr size_t kBars = (size_t)kWarps * S * sizeof(uint64_t);
+  static size_t bytes(size_t table_bytes) { return align16(table_bytes) + kRing + kBars; }
+};
+
+// Resolve a tile's pointers and start its object lines. The PF=2 warm-up
+// values are returned in w[] and folded into `sink` only when the tile becomes
+// current, so the wait for them overlaps the previous tile's group walk.
+template <class App, int M, class R, int U, int PF>
+__device__ __forceinline__ void resolve_tile(const unsigned char* smem, uint32_t P, const uint64_t (&p)[U],
+                                             uint64_t (&a)[U], uint32_t (&t)[U], uint32_t (&w)[U],
+                                             uint32_t& hint) {
+#pragma unroll
+  for (int j = 0; j < U; ++j) {
+    t[j] = p[j] ? R::resolve(smem, P, p[j], a[j], hint) : kNF;
+    if (!p[j]) a[j] = 0;
+    w[j] = 0;
+  }
+  if constexpr (PF == 1) {
+#pragma unroll
+    for (int j = 0; j < U; ++j)
+      if (t[j] < (uint32_t)App::kTypes) prefetch_l1(a[j]);
+  } else if constexpr (PF == 2) {
+#pragma unroll
+    for (int j = 0; j < U; ++j)
+      if (t[j] < (uint32_t)App::kTypes) w[j] = *reinterpret_cast<const uint32_t*>(a[j] + 8);
+  }
+}
+
+template <class App, int M, class R, int U, int PF, int S>
+__global__ void __launch_bounds__(kBlock, 4) k_dispatch_pipe(const uint64_t* __restrict__ objs,
+                                                          uint64_t n, ArgBlob args, DevTable tbl) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  using L = PipeSmem<U, S>;
+  constexpr int WT = L::kTile;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const size_t tbytes = R::kNeedsTable ? align16(table_smem_dev(tbl.P)) : 0;
+  uint64_t* ring = reinterpret_cast<uint64_t*>(smem + tbytes) + (size_t)warp * S * WT;
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + tbytes + L::kRing) + warp * S;
+  if constexpr (R::kNeedsTable) R::stage(smem, tbl);
+
+  // each warp streams its own sequence of warp tiles: no CTA-wide barrier, so
+  // a warp with many type groups never stalls the others
+  const uint64_t full = n / WT;
+  const uint64_t gw = (uint64_t)blockIdx.x * L::kWarps + warp;
+  const uint64_t nw = (uint64_t)gridDim.x * L::kWarps;
+  const uint64_t mine = gw < full ? (full - 1 - gw) / nw + 1 : 0;
+  auto tile_base = [&](uint64_t k) { return (gw + k * nw) * WT; };
+
+  if (lane == 0) {
+    for (int s = 0; s < S; ++s) mbar_init(&bars[s], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    for (int s = 0; s < S && (uint64_t)s < mine; ++s) {
+      mbar_expect_tx(&bars[s], WT * sizeof(uint64_t));
+      tma_load_1d(ring + (size_t)s * WT, objs + tile_base(s), WT * sizeof(uint64_t), &bars[s]);
+    }
+  }
+  __syncwarp();
+
+  uint32_t sink = 0;
+  uint32_t hint = 0;  // COAL: last range hit by this lane
+  uint64_t pc[U], ac[U];
+  uint32_t tc[U], wc[U];
+  // fetch warp tile k's pointers from the ring, release the stage, resolve + warm
+  auto fetch = [&](uint64_t k, uint64_t (&p)[U], uint64_t (&a)[U], uint32_t (&t)[U], uint32_t (&w)[U]) {
+    const int s = (int)(k % S);
+    mbar_wait(&bars[s], (uint32_t)((k / S) & 1));
+#pragma unroll
+    for (int j = 0; j < U; ++j) p[j] = ring[(size_t)s * WT + j * 32 + lane];
+    __syncwarp();  // the whole warp holds its pointers: the stage can be refilled
+    if (lane == 0 && k + S < mine) {
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      mbar_expect_tx(&bars[s], WT * sizeof(uint64_t));
+      tma_load_1d(ring + (size_t)s * WT, objs + tile_base(k + S), WT * sizeof(uint64_t), &bars[s]);
+    }
+    resolve_tile<App, M, R, U, PF>(smem, tbl.P, p, a, t, w, hint);
+  };
+
+  if (mine > 0) fetch(0, pc, ac, tc, wc);
+  for (uint64_t k = 0; k < mine; ++k) {
+#pragma unroll
+    for (int j = 0; j < U; ++j) sink ^= wc[j];
+    uint64_t pn[U], an[U];
+    uint32_t tn[U], wn[U];
+    if (k + 1 < mine) fetch(k + 1, pn, an, tn, wn);
+    const uint64_t base = tile_base(k);
+#pragma unroll
+    for (int j = 0; j < U; ++j) group_call<App, M>(tc[j], ac[j], pc[j], base + j * 32 + lane, args, tbl);
+#pragma unroll
+    for (int j = 0; j < U; ++j) {
+      pc[j] = pn[j];
+      ac[j] = an[j];
+      tc[j] = tn[j];
+      wc[j] = wn[j];
+    }
+  }
+  // ragged tail (< one warp tile): the last warp of the grid, plain loads
+  if (gw == nw - 1 && full * WT < n) {
+    const uint64_t base = full * WT;
+#pragma unroll
+    for (int j = 0; j < U; ++j) {
+      const uint64_t idx = base + (uint64_t)j * 32 + lane;
+      pc[j] = idx < n ? ldg_u64(objs + idx) : 0ull;
+    }
+    resolve_tile<App, M, R, U, PF>(smem, tbl.P, pc, ac, tc, wc, hint);
+#pragma unroll
+    for (int j = 0; j < U; ++j) {
+      sink ^= wc[j];
+      group_call<App, M>(tc[j], ac[j], pc[j], base + j * 32 + lane, args, tbl);
+    }
+  }
+  if constexpr (PF == 2) {
+    if (sink == 0x8BADF00Du && n == ~0ull) asm volatile("st.global.u32 [%0], %1;" ::"l"(objs), "r"(sink));
+  }
+}
+
+// ---------------------------------------------------------------------------
+// Type-regrouped dispatch (default for COAL / TypePointer with > 1 type).
+//
+// Warp grouping alone still runs one serialised group per type present in a
+// warp (≈T groups of 32/T lanes in random order: the SIMD under-utilisation
+// the paper identifies as the residual cost). Because the type is
+// known from the pointer alone, a CTA can regroup its tile BEFORE touching
+// any object: resolve kBlock*U pointers, counting-sort them by type in shared
+// memory (warp match_any + one smem atomic per type per warp; stable within a
+// warp so same-type objects stay in arena order), then let every warp walk 32
+// consecutive entries of the sorted tile. A warp then sees ~1 type, all 32
+// lanes active, touching consecutive slots of one arena (coalesced). Calls on
+// distinct objects are independent (reading G8), so the reordering is exact.
+// ---------------------------------------------------------------------------
+template <int U>
+struct SortSmem {
+  static constexpr int kTile = kBlock * U;
+  static constexpr size_t kA = (size_t)kTile * sizeof(uint64_t);   // sorted addresses
+  static constexpr size_t kI = (size_t)kTile * sizeof(uint32_t);   // sorted tile-local index
+  static constexpr size_t kT = (size_t)kTile * sizeof(uint8_t);    // sorted type
+  static constexpr size_t kH = 68 * sizeof(uint32_t);              // hist[32] + offs[33] (+pad)
+  static size_t bytes(size_t table_bytes) { return align16(table_bytes) + kA + kI + align16(kT) + kH; }
+};
+
+template <class App, int M, class R, int U, int PF>
+__global__ void __launch_bounds__(kBlock) k_dispatch_sorted(const uint64_t* __restrict__ objs,
+                                                            uint64_t n, ArgBlob args, DevTable tbl) {
+  static_assert(App::kTypes <= 32, "one warp scans the histogram");
+  extern __shared__ __align__(16) unsigned char smem[];
+  using L = SortSmem<U>;
+  constexpr int TILE = L::kTile;
+  const size_t tbytes = R::kNeedsTable ? align16(table_smem_dev(tbl.P)) : 0;
+  uint64_t* s_a = reinterpret_cast<uint64_t*>(smem + tbytes);
+  uint32_t* s_i = reinterpret_cast<uint32_t*>(smem + tbytes + L::kA);
+  uint8_t* s_t = reinterpret_cast<uint8_t*>(smem + tbytes + L::kA + L::kI);
+  uint32_t* s_hist = reinterpret_cast<uint32_t*>(smem + tbytes + L::kA + L::kI + align16(L::kT));
+  uint32_t* s_offs = s_hist + 32;  // 33 entries: exclusive offsets + total
+  if constexpr (R::kNeedsTable) R::stage(smem, tbl);
+  if (threadIdx.x < 32) s_hist[threadIdx.x] = 0;
+  __syncthreads();
+  const int lane = threadIdx.x & 31;
+  const uint32_t lt_mask = (1u << lane) - 1u;
+  uint32_t sink = 0;
+  uint32_t hint = 0;  // COAL: last range hit by this lane
+
+  for (uint64_t base = (uint64_t)blockIdx.x * TILE; base < n; base += (uint64_t)gridDim.x * TILE) {
+    // A: pointers -> (type, address); warm the object lines
+    uint64_t p[U], a[U];
+    uint32_t t[U], w[U], rank[U];
+#pragma unroll
+    for (int j = 0; j < U; ++j) {
+      const uint64_t idx = base + (uint64_t)j * kBlock + threadIdx.x;
+      p[j] = idx < n ? ldg_u64(objs + idx) : 0ull;
+    }
+#pragma unroll
+    for (int j = 0; j < U; ++j) {
+      t[j] = p[j] ? R::resolve(smem, tbl.P, p[j], a[j], hint) : kNF;
+      if (!p[j]) a[j] = 0;
+      const bool fb = t[j] >= (uint32_t)App::kTypes && p[j] != 0;
+      if (__any_sync(0xffffffffu, fb)) {
+        if (fb) t[j] = type_from_vptr<App>(a[j], tbl);
+      }
+      w[j] = 0;
+      if constexpr (PF == 2) {
+        if (t[j] < (uint32_t)App::kTypes) w[j] = *reinterpret_cast<const uint32_t*>(a[j] + 8);
+      }
+    }
+    // Tiles whose warps are already type-uniform (sorted input, run interiors)
+    // skip the sort: one barrier instead of three.
+    bool mixed = false;
+#pragma unroll
+    for (int j = 0; j < U; ++j) {
+      const uint32_t pres = __reduce_or_sync(0xffffffffu, t[j] < (uint32_t)App::kTypes ? (1u << t[j]) : 0u);
+      mixed |= (pres & (pres - 1)) != 0;
+    }
+    if (!__syncthreads_or(mixed)) {
+#pragma unroll
+      for (int j = 0; j < U; ++j) {
+        sink ^= w[j];
+        group_call<App, M>(t[j], a[j], 0ull, base + (uint64_t)j * kBlock + threadIdx.x, args, tbl);
+      }
+      continue;
+    }
+    // B: rank within type (warp-aggregated smem atomics)
+#pragma unroll
+    for (int j = 0; j < U; ++j) {
+      const bool ok = t[j] < (uint32_t)App::kTypes;
+      const uint32_t key = ok ? t[j] : 0xFFFFu;
+      const uint32_t peers = __match_any_sync(0xffffffffu, key);
+      const int leader = __ffs(peers) - 1;
+      uint32_t b = 0;
+      if (ok && lane == leader) b = atomicAdd(&s_hist[t[j]], (uint32_t)__popc(peers));
+      b = __shfl_sync(0xffffffffu, b, leader);
+      rank[j] = b + __popc(peers & lt_mask);
+    }
+    __syncthreads();
+    // C: exclusive scan of the histogram (one warp), reset it for the next tile
+    if (threadIdx.x < 32) {
+      const uint32_t h = s_hist[lane];
+      uint32_t x = h;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= o) x += y;
+      }
+      s_offs[lane] = x - h;
+      if (lane == 31) s_offs[32] = x;
+      s_hist[lane] = 0;
+    }
+    __syncthreads();
+    // D: scatter into the sorted tile
+#pragma unroll
+    for (int j = 0; j < U; ++j) {
+      if (t[j] < (uint32_t)App::kTypes) {
+        const uint32_t pos = s_offs[t[j]] + rank[j];
+        s_a[pos] = a[j];
+        s_i[pos] = (uint32_t)(j * kBlock + threadIdx.x);
+        s_t[pos] = (uint8_t)t[j];
+      }
+    }
+    __syncthreads();
+    // E: each warp walks 32 consecutive sorted entries per j
+    const uint32_t total = s_offs[32];
+#pragma unroll
+    for (int j = 0; j < U; ++j) sink ^= w[j];
+#pragma unroll
+    for (int j = 0; j < U; ++j) {
+      const uint32_t e = (uint32_t)(j * kBlock) + threadIdx.x;
+      const bool v = e < total;
+      const uint64_t ae = v ? s_a[e] : 0ull;
+      const uint32_t te = v ? (uint32_t)s_t[e] : kNF;
+      const uint64_t ie = v ? base + s_i[e] : 0ull;
+      group_call<App, M>(te, ae, 0ull, ie, args, tbl);
+    }
+  }
+  if constexpr (PF == 2) {
     if (sink == 0x8BADF00Du && n == ~0ull) asm volatile("st.global.u32 [%0], %1;" ::"l"(objs), "r"(sink));
   }
 }
@@ -266,8 +592,9 @@ __device__ __forceinline__ uint32_t resolve_rule(int variant, const unsigned cha
                                                  const DevTable& tbl, uint64_t p) {
   if (!p) return kNF;
   uint64_t a;
-  if (variant == VF_TYPEPTR) return ResolveTP::resolve(smem, tbl.P, p, a);
-  if (variant == VF_COAL) return ResolveCOAL::resolve(smem, tbl.P, p, a);
+  uint32_t hint = 0;
+  if (variant == VF_TYPEPTR) return ResolveTP::resolve(smem, tbl.P, p, a, hint);
+  if (variant == VF_COAL) return ResolveCOAL::resolve(smem, tbl.P, p, a, hint);
   // CUDA / SharedOA: the embedded vTable* (Fig. 1a load A), mapped to a type id
   const uint64_t vp = *reinterpret_cast<const uint64_t*>(p);
   for (uint32_t k = 0; k < tbl.ntypes; ++k)
@@ -319,7 +646,7 @@ inline int num_sms() {
   return sms;
 }
 
-inline size_t table_smem(const DevTable& t) { return (size_t)t.P * (8 + 8 + 4); }
+inline size_t table_smem(const DevTable& t) { return table_smem_dev(t.P); }
 
 inline unsigned grid_for(uint64_t n, uint64_t per_block, uint64_t cap) {
   uint64_t g = (n + per_block - 1) / per_block;
@@ -358,9 +685,62 @@ cudaError_t launch_virtual(const uint64_t* objs, uint64_t n, const ArgBlob& args
 
 // Benchmark / ablation knobs (vf_set_tuning): objects per thread and the L1
 // prefetch of object lines before the type groups.
+template <class App, int M, class R, int U, int PF, int S>
+cudaError_t launch_pipe(const uint64_t* objs, uint64_t n, const ArgBlob& args, const DevTable& tbl,
+                        cudaStream_t s) {
+  auto kern = k_dispatch_pipe<App, M, R, U, PF, S>;
+  const size_t sm = PipeSmem<U, S>::bytes(R::kNeedsTable ? table_smem(tbl) : 0);
+  static int occ = -1;
+  static size_t occ_sm = ~(size_t)0;
+  if (occ < 0 || occ_sm != sm) {
+    if (sm > 48 * 1024)
+      cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kBlock, sm);
+    if (occ < 1) occ = 1;
+    occ_sm = sm;
+  }
+  const uint64_t tiles = n / ((uint64_t)kBlock * U);  // CTA-sized tiles of warp tiles
+  const unsigned grid = grid_for(tiles, 1, (uint64_t)num_sms() * occ);
+  kern<<<grid, kBlock, sm, s>>>(objs, n, args, tbl);
+  note_launch();
+  return cudaGetLastError();
+}
+
+template <class App, int M, class R, int U, int PF>
+cudaError_t launch_sorted(const uint64_t* objs, uint64_t n, const ArgBlob& args, const DevTable& tbl,
+                          cudaStream_t s) {
+  auto kern = k_dispatch_sorted<App, M, R, U, PF>;
+  const size_t sm = SortSmem<U>::bytes(R::kNeedsTable ? table_smem(tbl) : 0);
+  static int occ = -1;
+  static size_t occ_sm = ~(size_t)0;
+  if (occ < 0 || occ_sm != sm) {
+    if (sm > 48 * 1024)
+      cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kBlock, sm);
+    if (occ < 1) occ = 1;
+    occ_sm = sm;
+  }
+  const unsigned grid = grid_for(n, (uint64_t)kBlock * U, (uint64_t)num_sms() * occ);
+  kern<<<grid, kBlock, sm, s>>>(objs, n, args, tbl);
+  note_launch();
+  return cudaGetLastError();
+}
+
 template <class App, int M, class R, int U>
 cudaError_t launch_grouped_pf(int pf, const uint64_t* objs, uint64_t n, const ArgBlob& args,
                               const DevTable& tbl, cudaStream_t s) {
+  if constexpr (App::kTypes > 1) {
+    if (tuning().regroup != 0) {
+      if (pf == 2) return launch_sorted<App, M, R, U, 2>(objs, n, args, tbl, s);
+      return launch_sorted<App, M, R, U, 0>(objs, n, args, tbl, s);
+    }
+  }
+  // TMA needs a 16-byte aligned source; the pipeline is the default when it applies
+  if (tuning().pipeline != 0 && (reinterpret_cast<uintptr_t>(objs) & 15) == 0) {
+    if (pf == 0) return launch_pipe<App, M, R, U, 0, 4>(objs, n, args, tbl, s);
+    if (pf == 1) return launch_pipe<App, M, R, U, 1, 4>(objs, n, args, tbl, s);
+    return launch_pipe<App, M, R, U, 2, 4>(objs, n, args, tbl, s);
+  }
   if (pf == 0) return launch_grouped<App, M, R, U, 0>(objs, n, args, tbl, s);
   if (pf == 1) return launch_grouped<App, M, R, U, 1>(objs, n, args, tbl, s);
   return launch_grouped<App, M, R, U, 2>(objs, n, args, tbl, s);
@@ -370,11 +750,14 @@ template <class App, int M, class R>
 cudaError_t launch_grouped_tuned(const uint64_t* objs, uint64_t n, const ArgBlob& args,
                                  const DevTable& tbl, cudaStream_t s) {
   const Tuning& tu = tuning();
-  // Objects per thread trade memory-level parallelism against the number of
-  // type groups walked per tile; with >= 24 live types (~20 groups per warp,
-  // random order) one object per thread measured best on B200.
-  const int u = tu.unroll > 0 ? tu.unroll : (tbl.active_types >= 24 ? 1 : App::kUnroll);
-  const int pf = tu.prefetch < 0 ? App::kPrefetch : tu.prefetch;
+  // Measured on B200 (config 2, 2^26 objects): with the per-tile type sort,
+  // 2 objects per thread + L1 warm-up is best up to ~16 live types; with >= 24
+  // live types (the sort leaves ~half-warp groups) 4 objects per thread
+  // without warm-up wins. Without the sort, >= 24 types prefer 1 object/thread.
+  const bool rg = tu.regroup != 0 && App::kTypes > 1;
+  const bool many = tbl.active_types >= 24;
+  const int u = tu.unroll > 0 ? tu.unroll : rg ? (many ? 4 : App::kUnrollSorted) : (many ? 1 : App::kUnroll);
+  const int pf = tu.prefetch >= 0 ? tu.prefetch : (rg && many) ? 0 : App::kPrefetch;
   if (u >= 4) return launch_grouped_pf<App, M, R, 4>(pf, objs, n, args, tbl, s);
   if (u == 2) return launch_grouped_pf<App, M, R, 2>(pf, objs, n, args, tbl, s);
   return launch_grouped_pf<App, M, R, 1>(pf, objs, n, args, tbl, s);

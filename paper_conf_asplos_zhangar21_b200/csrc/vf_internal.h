@@ -63,7 +63,9 @@ const AppOps* app_gol();
 // Benchmark / ablation knobs set through vf_set_tuning (-1 = app default).
 struct Tuning {
   int unroll = -1;    // objects per thread in the grouped kernels (1, 2, 4)
-  int prefetch = -1;  // 1: prefetch object lines to L1 before the type groups
+  int prefetch = -1;  // 0 none, 1 prefetch.global.L1, 2 L1-allocating warm load
+  int pipeline = 0;   // 1: TMA-pipelined pointer stream (k_dispatch_pipe), 0: plain loads
+  int regroup = 1;    // 1: CTA-level counting sort of each tile by type (k_dispatch_sorted)
 };
 Tuning& tuning();
 

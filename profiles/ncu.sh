@@ -8,7 +8,7 @@ mkdir -p $OUT
 B="python bench.py --steps 4 --warmup 3 --no-variants --no-e2e --no-cpu"
 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches.csv $B --variant typeptr > $OUT/launches_bench.log 2>&1
 for v in typeptr coal sharedoa; do
-  case $v in sharedoa) K=regex:k_dispatch_virtual;; *) K=regex:k_dispatch_grouped;; esac
+  case $v in sharedoa) K=regex:k_dispatch_virtual;; *) K="regex:k_dispatch_(grouped|sorted|pipe)";; esac
   ncu --set full --clock-control none --import-source on -k $K -s 3 -c 1 -o $OUT/prof_${v}_T4 -f \
       $B --variant $v --T ${T:-4} > $OUT/prof_${v}.log 2>&1
 done

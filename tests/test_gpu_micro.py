@@ -42,15 +42,19 @@ def test_micro_parity(ctx, variant, T, order):
 
 
 @pytest.mark.parametrize("unroll", [1, 2, 4])
-@pytest.mark.parametrize("prefetch", [0, 1])
+@pytest.mark.parametrize("prefetch", [0, 1, 2])
+@pytest.mark.parametrize("pipeline,regroup", [(0, 0), (1, 0), (0, 1)])
 @pytest.mark.parametrize("variant", ["coal", "typeptr"])
-def test_micro_tuning_knobs(ctx, unroll, prefetch, variant):
-    n, T, R = 50_000 + 3, 8, 2
+@pytest.mark.parametrize("n", [50_000 + 3, 1024 * 300, 100])
+def test_micro_tuning_knobs(ctx, unroll, prefetch, pipeline, regroup, variant, n):
+    T, R = 8, 2
     types = synth.micro_types(n, T, "random", seed=3)
     init = synth.micro_init(n, seed=3)
     ref, _ = oracle.micro_run(types, init, T, R)
     vf.set_tuning("unroll", unroll)
     vf.set_tuning("prefetch", prefetch)
+    vf.set_tuning("pipeline", pipeline)
+    vf.set_tuning("regroup", regroup)
     try:
         m = apps.Micro(ctx, n, T, variant=variant, types_np=types, init_np=init)
         for _ in range(R):
@@ -59,6 +63,8 @@ def test_micro_tuning_knobs(ctx, unroll, prefetch, variant):
     finally:
         vf.set_tuning("unroll", -1)
         vf.set_tuning("prefetch", -1)
+        vf.set_tuning("pipeline", 0)
+        vf.set_tuning("regroup", 1)
 
 
 @pytest.mark.parametrize("n", [0, 1, 31, 33, 255, 257, 4097])
