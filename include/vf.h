@@ -63,7 +63,8 @@ typedef enum { VF_CUDA = 0, VF_SHAREDOA = 1, VF_COAL = 2, VF_TYPEPTR = 3 } vf_va
 enum {
   VF_APP_MICRO = 0, /* config 2: MObj<k>::apply(){ val += k+1; }  (§8.3)      */
   VF_APP_GOL = 1,   /* config 1: Cell / Alive / Dead               (Table 2)  */
-  VF_APP_COUNT = 2
+  VF_APP_GEN = 2,   /* config 5: Cell / Dead / Alive / Dying       (Table 2)  */
+  VF_APP_COUNT = 3
 };
 
 /* Methods of VF_APP_MICRO (args structs are passed by value, see dispatch). */
@@ -79,6 +80,17 @@ typedef struct {
   uint8_t* state_out_dev;   /* next state per cell                                          */
 } vf_gol_next_args;
 typedef struct { uint16_t* counter_out_dev; uint8_t* type_out_dev; } vf_gol_get_args;
+
+/* Methods of VF_APP_GEN (Generations CA B/S/C, reading G15; type ids 0 Dead,
+ * 1 Alive, 2 Dying). born/survive: bit n set = rule holds with n live
+ * (state-1) neighbours; C = number of states (2..255). */
+enum { VF_GEN_NEXT = 0, VF_GEN_GET = 1 };
+typedef struct {
+  const uint8_t* nbr_dev;   /* live (state-1) neighbours per cell                  */
+  uint8_t* state_out_dev;   /* next state per cell                                 */
+  uint32_t born_mask, survive_mask, C;
+} vf_gen_next_args;
+typedef struct { uint16_t* counter_out_dev; uint8_t* type_out_dev; } vf_gen_get_args;
 
 #define VF_MAX_RANGES 4096u     /* COAL range-table capacity (staged in shared memory)   */
 #define VF_MAX_ARGS_BYTES 256u  /* method argument blob, copied into kernel parameters   */
@@ -201,8 +213,8 @@ vf_status vf_dispatch(vf_ctx* ctx, vf_variant v, uint32_t app, uint32_t method,
                       void* stream);
 
 /* ---- app helpers (non-virtual phases) ---------------------------------- */
-/* GOL step (1): nbr_dev[c] = live neighbours of cell c in state_dev (W x H,
- * dead border, or torus if torus != 0). */
+/* GOL / GEN step (1): nbr_dev[c] = neighbours of cell c whose state is 1
+ * (alive) in state_dev (W x H, dead border, or torus if torus != 0). */
 vf_status vf_gol_neighbors(uint32_t W, uint32_t H, int torus, const uint8_t* state_dev,
                            uint8_t* nbr_dev, void* stream);
 /* GOL step (3): where state_next != state_prev, swap grid_dev[c] between
@@ -210,6 +222,12 @@ vf_status vf_gol_neighbors(uint32_t W, uint32_t H, int torus, const uint8_t* sta
 vf_status vf_gol_swap(vf_ctx* ctx, uint64_t ncells, const uint8_t* state_prev_dev,
                       const uint8_t* state_next_dev, uint64_t* grid_dev,
                       const uint64_t* alive_dev, const uint64_t* dead_dev, void* stream);
+/* GEN step (3): where the type of state_next differs from state_prev's, point
+ * grid_dev[c] at the cell's Dead / Alive / Dying object, reset its counter and
+ * (Dying) set its stage to the new state. */
+vf_status vf_gen_swap(vf_ctx* ctx, uint64_t ncells, const uint8_t* state_prev_dev,
+                      const uint8_t* state_next_dev, uint64_t* grid_dev, const uint64_t* dead_dev,
+                      const uint64_t* alive_dev, const uint64_t* dying_dev, void* stream);
 
 /* ---- utilities ---------------------------------------------------------- */
 /* sum over i of vals_dev[i] (int32, widened) into *out_dev (i64, device). */

@@ -27,7 +27,7 @@ import numpy as np
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 SO = os.path.join(HERE, "liboracle.so")
-SOURCES = ["alloc.cpp", "micro.cpp", "gol.cpp"]
+SOURCES = ["alloc.cpp", "micro.cpp", "gol.cpp", "gen.cpp", "graph.cpp"]
 NOT_FOUND = 0xFFFFFFFF
 
 
@@ -76,6 +76,19 @@ def lib():
         L.oracle_gol_run.argtypes = [ctypes.c_uint32, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_uint32,
                                      ctypes.c_int, ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p,
                                      ctypes.c_void_p, ctypes.POINTER(ctypes.c_double)]
+        L.oracle_gen_run.restype = ctypes.c_int
+        L.oracle_gen_run.argtypes = [ctypes.c_uint32, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_uint32,
+                                     ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_int,
+                                     ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
+                                     ctypes.POINTER(ctypes.c_double)]
+        P, U32, U64 = ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint64
+        L.oracle_graph_bfs.restype = ctypes.c_int
+        L.oracle_graph_bfs.argtypes = [U64, P, P, P, U32, P, P, P, ctypes.POINTER(ctypes.c_double)]
+        L.oracle_graph_cc.restype = ctypes.c_int
+        L.oracle_graph_cc.argtypes = [U64, P, P, P, ctypes.c_int, P, P, P, ctypes.POINTER(ctypes.c_double)]
+        L.oracle_graph_pr.restype = ctypes.c_int
+        L.oracle_graph_pr.argtypes = [U64, P, P, P, ctypes.c_double, U32, ctypes.c_int, P,
+                                      ctypes.POINTER(ctypes.c_double)]
         L.oracle_max_threads.restype = ctypes.c_int
         _lib = L
     return _lib
@@ -168,3 +181,68 @@ def gol_run(W: int, H: int, alive0, gens: int, torus: bool = False, threads: int
     if rc != 0:
         raise ValueError(f"oracle_gol_run rc={rc}")
     return st, ctr, pop[:gens].copy(), sec.value
+
+
+def rule_masks(born, survive):
+    """'B2/S345' style digit strings -> bit masks."""
+    return sum(1 << int(d) for d in str(born)), sum(1 << int(d) for d in str(survive))
+
+
+def gen_run(W: int, H: int, state0, gens: int, born="2", survive="345", C: int = 4,
+            torus: bool = False, threads: int = 1):
+    """Returns (state uint8[H*W], counter uint16[H*W], hist uint32[C], seconds)."""
+    bm, sm = rule_masks(born, survive)
+    a = np.ascontiguousarray(state0, dtype=np.uint8)
+    st = np.zeros(W * H, np.uint8)
+    ctr = np.zeros(W * H, np.uint16)
+    hist = np.zeros(C, np.uint32)
+    sec = ctypes.c_double(0.0)
+    rc = lib().oracle_gen_run(W, H, a.ctypes.data, gens, bm, sm, C, int(torus), threads, st.ctypes.data,
+                              ctr.ctypes.data, hist.ctypes.data, ctypes.byref(sec))
+    if rc != 0:
+        raise ValueError(f"oracle_gen_run rc={rc}")
+    return st, ctr, hist, sec.value
+
+
+def _csr(offs, col, types):
+    return (np.ascontiguousarray(offs, dtype=np.uint64), np.ascontiguousarray(col, dtype=np.uint32),
+            np.ascontiguousarray(types, dtype=np.uint32))
+
+
+def graph_bfs(offs, col, types, src: int):
+    """Returns (depth int32[V], levels, calls, seconds)."""
+    offs, col, types = _csr(offs, col, types)
+    V = len(offs) - 1
+    depth = np.empty(V, np.int32)
+    lv, calls, sec = ctypes.c_uint32(), ctypes.c_uint64(), ctypes.c_double()
+    rc = lib().oracle_graph_bfs(V, offs.ctypes.data, col.ctypes.data, types.ctypes.data, src,
+                                depth.ctypes.data, ctypes.byref(lv), ctypes.byref(calls), ctypes.byref(sec))
+    if rc:
+        raise ValueError(f"oracle_graph_bfs rc={rc}")
+    return depth, lv.value, calls.value, sec.value
+
+
+def graph_cc(offs, col, types, threads: int = 1):
+    """Returns (label uint32[V], iters, calls, seconds)."""
+    offs, col, types = _csr(offs, col, types)
+    V = len(offs) - 1
+    label = np.empty(V, np.uint32)
+    it, calls, sec = ctypes.c_uint32(), ctypes.c_uint64(), ctypes.c_double()
+    rc = lib().oracle_graph_cc(V, offs.ctypes.data, col.ctypes.data, types.ctypes.data, threads,
+                               label.ctypes.data, ctypes.byref(it), ctypes.byref(calls), ctypes.byref(sec))
+    if rc:
+        raise ValueError(f"oracle_graph_cc rc={rc}")
+    return label, it.value, calls.value, sec.value
+
+
+def graph_pr(offs, col, types, iters: int = 20, d: float = 0.85, threads: int = 1):
+    """Returns (rank float32[V], seconds)."""
+    offs, col, types = _csr(offs, col, types)
+    V = len(offs) - 1
+    rank = np.empty(V, np.float32)
+    sec = ctypes.c_double()
+    rc = lib().oracle_graph_pr(V, offs.ctypes.data, col.ctypes.data, types.ctypes.data, d, iters, threads,
+                               rank.ctypes.data, ctypes.byref(sec))
+    if rc:
+        raise ValueError(f"oracle_graph_pr rc={rc}")
+    return rank, sec.value

@@ -89,6 +89,39 @@ int oracle_gol_run(uint32_t W, uint32_t H, const uint8_t* init_alive,
                    uint8_t* out_state, uint16_t* out_counter, uint32_t* pop,
                    double* seconds);
 
+/* ---- Config 5 Generation (Table 2; reading G15) ------------
+ * Generations CA B/S/C: states 0 dead, 1 alive, 2..C-1 dying. born_mask /
+ * survive_mask bit n = rule holds with n live (state-1) neighbours. Per
+ * generation: n[c] from the previous state (dead border / torus), one virtual
+ * next() per cell (Dead: born? 1 : 0; Alive: survive? 1 : (C>2 ? 2 : 0);
+ * Dying(s): s+1 < C ? s+1 : 0), pointer swap on a type change. hist[k] =
+ * cells in state k at the end (C entries). */
+int oracle_gen_run(uint32_t W, uint32_t H, const uint8_t* init_state, uint32_t gens,
+                   uint32_t born_mask, uint32_t survive_mask, uint32_t C, int torus,
+                   int threads, uint8_t* out_state, uint16_t* out_counter, uint32_t* hist,
+                   double* seconds);
+
+/* ---- Config 4 graph apps over polymorphic vertices (Table 2 P:1538-1588;
+ * readings G20-G23). CSR offs[V+1] / col[arcs] (symmetric), types[v] in
+ * {0 Leaf, 1 Low, 2 Mid, 3 Hub}; one object per vertex from plain `new`.
+ * BFS: level-synchronous from src, one virtual bfs_expand() per frontier
+ *   vertex; depth[v] = level or -1; *levels = levels visited (incl. the
+ *   empty last), *calls = sum of frontier sizes.
+ * CC: Jacobi min-label propagation from label = id until no change, one
+ *   virtual cc_update() per vertex per iteration (*iters incl. the final
+ *   no-change pass).
+ * PR: r0 = 1/V; per iteration c_u = deg ? r_u/deg : 0 (fp64), D = sum of r
+ *   over deg-0 vertices (fp64, vertex order), s_v = virtual pr_gather() =
+ *   sum over N(v) of c_u in CSR order (fp64), r_v' = (float)((1-d)/V +
+ *   d*(s_v + D/V)). */
+int oracle_graph_bfs(uint64_t V, const uint64_t* offs, const uint32_t* col, const uint32_t* types,
+                     uint32_t src, int32_t* depth, uint32_t* levels, uint64_t* calls,
+                     double* seconds);
+int oracle_graph_cc(uint64_t V, const uint64_t* offs, const uint32_t* col, const uint32_t* types,
+                    int threads, uint32_t* label, uint32_t* iters, uint64_t* calls, double* seconds);
+int oracle_graph_pr(uint64_t V, const uint64_t* offs, const uint32_t* col, const uint32_t* types,
+                    double d, uint32_t iters, int threads, float* rank, double* seconds);
+
 /* number of OpenMP threads actually available */
 int oracle_max_threads(void);
 

@@ -110,3 +110,58 @@ class Gol:
         self.ctx.dispatch(self.v, vf.APP_GOL, vf.GOL_GET, self.grid,
                           vf.gol_get_args(ctr.data_ptr(), typ.data_ptr()))
         return ctr, typ
+
+
+def rule_masks(born: str, survive: str):
+    """'B2/S345' digit strings -> (born_mask, survive_mask)."""
+    return sum(1 << int(d) for d in str(born)), sum(1 << int(d) for d in str(survive))
+
+
+class Gen:
+    """Config 5 GEN: Generations CA B/S/C over polymorphic Dead / Alive / Dying cells
+    (Table 2, reading G15). Same three steps per generation as Gol."""
+
+    def __init__(self, ctx: vf.Ctx, W: int, H: int, state0, variant: str = "typeptr",
+                 born: str = "2", survive: str = "345", C: int = 4, torus: bool = False):
+        self.ctx, self.W, self.H, self.variant, self.torus = ctx, W, H, variant, torus
+        self.v = vf.VARIANTS[variant]
+        dev = _dev(ctx.device)
+        N = W * H
+        self.N = N
+        cells = torch.arange(N, dtype=torch.int32, device=dev)
+        objs = []
+        for t in range(3):
+            if variant == "cuda":
+                objs.append(ctx.alloc_cuda(vf.APP_GEN, torch.full((N,), t, dtype=torch.int32, device=dev), cells))
+            else:
+                objs.append(ctx.alloc_typed(vf.APP_GEN, t, N, cells, tag=(variant == "typeptr")))
+        self.dead, self.alive, self.dying = objs
+        self.grid = self.dead.clone()
+        s0 = torch.from_numpy(np.ascontiguousarray(state0, dtype=np.uint8)).to(dev)
+        zeros = torch.zeros(N, dtype=torch.uint8, device=dev)
+        vf.gen_swap(ctx, zeros, s0, self.grid, self.dead, self.alive, self.dying)
+        self.state = s0.clone()
+        self.next = torch.empty_like(self.state)
+        self.nbr = torch.empty_like(self.state)
+        bm, sm = rule_masks(born, survive)
+        self.args = [vf.gen_next_args(self.nbr.data_ptr(), self.next.data_ptr(), bm, sm, C),
+                     vf.gen_next_args(self.nbr.data_ptr(), self.state.data_ptr(), bm, sm, C)]
+        self.parity = 0
+        torch.cuda.synchronize(dev)
+
+    def gen(self, stream=None):
+        cur, nxt = (self.state, self.next) if self.parity == 0 else (self.next, self.state)
+        vf.gol_neighbors(self.W, self.H, cur, self.nbr, self.torus, stream)
+        self.ctx.dispatch(self.v, vf.APP_GEN, vf.GEN_NEXT, self.grid, self.args[self.parity], stream=stream)
+        vf.gen_swap(self.ctx, cur, nxt, self.grid, self.dead, self.alive, self.dying, stream)
+        self.parity ^= 1
+
+    @property
+    def current(self):
+        return self.state if self.parity == 0 else self.next
+
+    def counters(self):
+        ctr = torch.empty(self.N, dtype=torch.int16, device=self.grid.device)
+        typ = torch.empty(self.N, dtype=torch.uint8, device=self.grid.device)
+        self.ctx.dispatch(self.v, vf.APP_GEN, vf.GEN_GET, self.grid, vf.gen_get_args(ctr.data_ptr(), typ.data_ptr()))
+        return ctr, typ

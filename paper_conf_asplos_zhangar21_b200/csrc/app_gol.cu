@@ -100,7 +100,7 @@ __global__ void k_neighbors(uint32_t W, uint32_t H, int torus, const uint8_t* __
       } else if (yy < 0 || yy >= (int)H || xx < 0 || xx >= (int)W) {
         continue;
       }
-      n += st[(uint64_t)yy * W + xx];
+      n += st[(uint64_t)yy * W + xx] == 1;
     }
   nb[c] = (uint8_t)n;
 }

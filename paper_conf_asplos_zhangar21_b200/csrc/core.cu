@@ -35,6 +35,7 @@ static const AppOps* app_ops(uint32_t app) {
   switch (app) {
     case VF_APP_MICRO: return app_micro();
     case VF_APP_GOL: return app_gol();
+    case VF_APP_GEN: return app_gen();
   }
   return nullptr;
 }

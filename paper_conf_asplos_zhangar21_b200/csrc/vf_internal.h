@@ -59,6 +59,7 @@ struct AppOps {
 
 const AppOps* app_micro();
 const AppOps* app_gol();
+const AppOps* app_gen();
 
 // Benchmark / ablation knobs set through vf_set_tuning (-1 = app default).
 struct Tuning {

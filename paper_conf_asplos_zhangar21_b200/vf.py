@@ -19,9 +19,10 @@ SO = os.path.join(PKG, "libvf.so")
 VF_OK = 0
 CUDA, SHAREDOA, COAL, TYPEPTR = 0, 1, 2, 3
 VARIANTS = {"cuda": CUDA, "sharedoa": SHAREDOA, "coal": COAL, "typeptr": TYPEPTR}
-APP_MICRO, APP_GOL = 0, 1
+APP_MICRO, APP_GOL, APP_GEN = 0, 1, 2
 MICRO_APPLY, MICRO_GET = 0, 1
 GOL_NEXT, GOL_GET = 0, 1
+GEN_NEXT, GEN_GET = 0, 1
 NOT_FOUND = 0xFFFFFFFF
 VA_BITS = 57
 MAX_RANGES = 4096
@@ -35,7 +36,7 @@ SYMBOLS = [
     "vf_alloc_typed", "vf_alloc_typed_batch", "vf_alloc_cuda", "vf_reset", "vf_range_table",
     "vf_regions", "vf_type_vptrs", "vf_resolve", "vf_verify_types", "vf_dispatch_cuda",
     "vf_dispatch_sharedoa", "vf_dispatch_coal", "vf_dispatch_typeptr", "vf_dispatch",
-    "vf_gol_neighbors", "vf_gol_swap", "vf_checksum_i32", "vf_launch_count", "vf_set_tuning",
+    "vf_gol_neighbors", "vf_gol_swap", "vf_gen_swap", "vf_checksum_i32", "vf_launch_count", "vf_set_tuning",
 ]
 
 
@@ -74,6 +75,14 @@ class gol_get_args(ctypes.Structure):
     _fields_ = [("counter_out_dev", ctypes.c_void_p), ("type_out_dev", ctypes.c_void_p)]
 
 
+class gen_next_args(ctypes.Structure):
+    _fields_ = [("nbr_dev", ctypes.c_void_p), ("state_out_dev", ctypes.c_void_p),
+                ("born_mask", ctypes.c_uint32), ("survive_mask", ctypes.c_uint32), ("C", ctypes.c_uint32)]
+
+
+gen_get_args = gol_get_args
+
+
 _lib = None
 
 
@@ -109,6 +118,7 @@ def lib(required: bool = True):
         "vf_dispatch_typeptr": (I, [P, U32, U32, P, U64, P, ctypes.c_size_t, P]),
         "vf_gol_neighbors": (I, [U32, U32, I, P, P, P]),
         "vf_gol_swap": (I, [P, U64, P, P, P, P, P, P]),
+        "vf_gen_swap": (I, [P, U64, P, P, P, P, P, P, P]),
         "vf_checksum_i32": (I, [P, U64, P, P]),
         "vf_launch_count": (U64, []),
         "vf_set_tuning": (I, [ctypes.c_char_p, I]),
@@ -295,6 +305,13 @@ def gol_swap(ctx: Ctx, prev, nxt, grid, alive, dead, stream=None):
                            _ptr(dead), _stream(stream))
     if st:
         raise VFError(st, "gol_swap")
+
+
+def gen_swap(ctx: Ctx, prev, nxt, grid, dead, alive, dying, stream=None):
+    st = lib().vf_gen_swap(ctx.h, grid.numel(), _ptr(prev), _ptr(nxt), _ptr(grid), _ptr(dead),
+                           _ptr(alive), _ptr(dying), _stream(stream))
+    if st:
+        raise VFError(st, "gen_swap")
 
 
 def checksum_i32(vals, out, stream=None):

@@ -131,3 +131,76 @@ def place(W: int, H: int, cells) -> np.ndarray:
     for x, y in cells:
         g[y * W + x] = 1
     return g
+
+
+# --------------------------------------------------------------------------
+# Config 4: RMAT graph. Native helper synth/rmat.cpp.
+# --------------------------------------------------------------------------
+_rmat_lib = None
+
+
+def _rmat():
+    global _rmat_lib
+    if _rmat_lib is None:
+        import ctypes
+        import os
+        import subprocess
+        here = os.path.dirname(os.path.abspath(__file__))
+        so, src = os.path.join(here, "libsynth.so"), os.path.join(here, "rmat.cpp")
+        if not os.path.exists(so) or os.path.getmtime(so) < os.path.getmtime(src):
+            subprocess.run(["g++", "-O2", "-std=c++17", "-fopenmp", "-fPIC", "-shared", "-o", so, src], check=True)
+        L = ctypes.CDLL(so)
+        P, U32, U64, D = ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_double
+        L.synth_rmat_edges.argtypes = [U32, U64, D, D, D, U64, U64, P, P]
+        L.synth_rmat_edges.restype = None
+        L.synth_permutation.argtypes = [U64, U64, U64, P]
+        L.synth_permutation.restype = None
+        L.synth_csr.argtypes = [U64, U64, P, P, P, P, P]
+        L.synth_csr.restype = U64
+        _rmat_lib = L
+    return _rmat_lib
+
+
+def build_native() -> None:
+    _rmat()
+
+
+def rmat_graph(scale: int, edge_factor: int = 16, seed: int = 1, A: float = 0.57, B: float = 0.19,
+               C: float = 0.19, permute: bool = True):
+    """Symmetric, de-duplicated, self-loop-free RMAT CSR: (offs uint64[V+1], col uint32[arcs])."""
+    L = _rmat()
+    V = 1 << scale
+    E = edge_factor * V
+    src = np.empty(E, np.uint32)
+    dst = np.empty(E, np.uint32)
+    L.synth_rmat_edges(scale, E, A, B, C, seed, S_GRAPH, src.ctypes.data, dst.ctypes.data)
+    perm = None
+    if permute:
+        perm = np.empty(V, np.uint32)
+        L.synth_permutation(V, seed, S_PERM, perm.ctypes.data)
+    offs = np.empty(V + 1, np.uint64)
+    col = np.empty(2 * E, np.uint32)
+    arcs = L.synth_csr(V, E, src.ctypes.data, dst.ctypes.data, None if perm is None else perm.ctypes.data,
+                       offs.ctypes.data, col.ctypes.data)
+    return offs, col[:arcs].copy()
+
+
+def csr_from_edges(V: int, edges):
+    """Symmetric CSR of a small explicit undirected edge list (fixtures)."""
+    L = _rmat()
+    e = np.asarray(edges, dtype=np.uint32).reshape(-1, 2)
+    src = np.ascontiguousarray(e[:, 0])
+    dst = np.ascontiguousarray(e[:, 1])
+    offs = np.empty(V + 1, np.uint64)
+    col = np.empty(max(2 * len(e), 1), np.uint32)
+    arcs = L.synth_csr(V, len(e), src.ctypes.data, dst.ctypes.data, None, offs.ctypes.data, col.ctypes.data)
+    return offs, col[:arcs].copy()
+
+
+# degree-bucket vertex types (SURVEY W6, reading G22): Leaf <=1, Low 2-15, Mid 16-255, Hub >=256
+DEG_BOUNDS = (1, 15, 255)
+
+
+def vertex_types(offs) -> np.ndarray:
+    deg = np.diff(np.asarray(offs, dtype=np.int64))
+    return np.digitize(deg, [DEG_BOUNDS[0] + 1, DEG_BOUNDS[1] + 1, DEG_BOUNDS[2] + 1]).astype(np.uint32)
