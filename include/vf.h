@@ -64,7 +64,8 @@ enum {
   VF_APP_MICRO = 0, /* config 2: MObj<k>::apply(){ val += k+1; }  (§8.3)      */
   VF_APP_GOL = 1,   /* config 1: Cell / Alive / Dead               (Table 2)  */
   VF_APP_GEN = 2,   /* config 5: Cell / Dead / Alive / Dying       (Table 2)  */
-  VF_APP_COUNT = 3
+  VF_APP_GRAPH = 3, /* config 4: Vertex / Leaf / Low / Mid / Hub   (Table 2)  */
+  VF_APP_COUNT = 4
 };
 
 /* Methods of VF_APP_MICRO (args structs are passed by value, see dispatch). */
@@ -91,6 +92,48 @@ typedef struct {
   uint32_t born_mask, survive_mask, C;
 } vf_gen_next_args;
 typedef struct { uint16_t* counter_out_dev; uint8_t* type_out_dev; } vf_gen_get_args;
+
+/* Methods of VF_APP_GRAPH (readings G20-G23). Type ids by degree: 0 Leaf
+ * (<= 1), 1 Low (2..15), 2 Mid (16..255), 3 Hub (>= 256). Constructor
+ * argument per object: { u32 vid, u32 deg }. CSR: offs[V+1] (u64), col (u32),
+ * symmetric. vobj_dev[v] = the object pointer of vertex v. */
+enum {
+  VF_GRAPH_BFS_EXPAND = 0, /* top-down: claim depth[u] = level+1 for unvisited neighbours
+                              (atomicCAS) and append vobj[u] to next_queue            */
+  VF_GRAPH_BFS_PROBE = 1,  /* bottom-up: an unvisited vertex with a neighbour at `level`
+                              takes depth level+1; next_count counts them               */
+  VF_GRAPH_CC_UPDATE = 2,  /* label_out[v] = min(label_in over v and N(v)); changed = 1
+                              if it differs from label_in[v] (Jacobi)                   */
+  VF_GRAPH_PR_CONTRIB = 3, /* contrib[v] = deg ? rank_in[v]/deg : 0 (fp64); deg-0
+                              vertices add rank_in[v] to *dangling                       */
+  VF_GRAPH_PR_UPDATE = 4   /* rank_out[v] = (float)(base + d*(sum_{N(v)} contrib +
+                              *dangling / Vd)), base = (1-d)/V                          */
+};
+typedef struct {
+  const uint64_t* offs_dev;
+  const uint32_t* col_dev;
+  int32_t* depth_dev;
+  const uint64_t* vobj_dev;
+  uint64_t* next_queue_dev;
+  uint32_t* next_count_dev;
+  int32_t level;
+} vf_graph_bfs_args;
+typedef struct {
+  const uint64_t* offs_dev;
+  const uint32_t* col_dev;
+  const uint32_t* label_in_dev;
+  uint32_t* label_out_dev;
+  uint32_t* changed_dev;
+} vf_graph_cc_args;
+typedef struct {
+  const uint64_t* offs_dev;
+  const uint32_t* col_dev;
+  const float* rank_in_dev;
+  float* rank_out_dev;
+  double* contrib_dev;
+  double* dangling_dev;
+  double base, d, Vd;
+} vf_graph_pr_args;
 
 #define VF_MAX_RANGES 4096u     /* COAL range-table capacity (staged in shared memory)   */
 #define VF_MAX_ARGS_BYTES 256u  /* method argument blob, copied into kernel parameters   */
@@ -228,6 +271,13 @@ vf_status vf_gol_swap(vf_ctx* ctx, uint64_t ncells, const uint8_t* state_prev_de
 vf_status vf_gen_swap(vf_ctx* ctx, uint64_t ncells, const uint8_t* state_prev_dev,
                       const uint8_t* state_next_dev, uint64_t* grid_dev, const uint64_t* dead_dev,
                       const uint64_t* alive_dev, const uint64_t* dying_dev, void* stream);
+
+/* Graph helpers: BFS start state (depth = -1 except depth[src] = 0, queue =
+ * [vobj[src]], *count = 1), iota (x[i] = i), fill (x[i] = value). */
+vf_status vf_graph_bfs_init(uint64_t V, int32_t* depth_dev, uint32_t src, const uint64_t* vobj_dev,
+                            uint64_t* queue_dev, uint32_t* count_dev, void* stream);
+vf_status vf_iota_u32(uint64_t n, uint32_t* x_dev, void* stream);
+vf_status vf_fill_f32(uint64_t n, float* x_dev, float value, void* stream);
 
 /* ---- utilities ---------------------------------------------------------- */
 /* sum over i of vals_dev[i] (int32, widened) into *out_dev (i64, device). */

@@ -1,0 +1,218 @@
+// app_graph.cu — config 4: BFS / CC / PageRank over polymorphic vertices
+// (Table 2 GraphChi apps; BASELINE north_star: polymorphic
+// vertices on a synthetic RMAT graph, reading G22). Vertex classes by degree
+// bucket: Leaf (deg <= 1), Low (2..15), Mid (16..255), Hub (>= 256). All four
+// implement the same semantics (the oracle's plain loops); each picks the
+// loop shape that suits its degree: Leaf has no loop, Low a plain loop, Mid
+// and Hub unrolled loops with independent accumulators (more loads in flight).
+//
+// Object layout (16 B): { vTable* (8 B), u32 vid, u32 deg }.
+#include "dispatch.cuh"
+
+namespace vf {
+namespace graph {
+
+struct CtorArg {
+  uint32_t vid, deg;
+};
+
+struct Vertex {
+  __device__ explicit Vertex(const void* arg)
+      : vid(arg ? static_cast<const CtorArg*>(arg)->vid : 0),
+        deg(arg ? static_cast<const CtorArg*>(arg)->deg : 0) {}
+  __device__ virtual ~Vertex() {}
+  __device__ virtual void bfs_expand(vf_graph_bfs_args a) = 0;
+  __device__ virtual void bfs_probe(vf_graph_bfs_args a) = 0;
+  __device__ virtual void cc_update(vf_graph_cc_args a) = 0;
+  __device__ virtual void pr_contrib(vf_graph_pr_args a) = 0;
+  __device__ virtual void pr_update(vf_graph_pr_args a) = 0;
+  uint32_t vid;
+  uint32_t deg;
+};
+
+// Neighbour loop with U independent lanes of work (U = 1: plain loop).
+template <int U, class F>
+__device__ __forceinline__ void for_neighbors(const uint32_t* __restrict__ col, uint64_t b, uint64_t e, F&& f) {
+  uint64_t k = b;
+  if constexpr (U > 1) {
+    for (; k + U <= e; k += U) {
+      uint32_t u[U];
+#pragma unroll
+      for (int j = 0; j < U; ++j) u[j] = __ldg(col + k + j);
+#pragma unroll
+      for (int j = 0; j < U; ++j) f(u[j]);
+    }
+  }
+  for (; k < e; ++k) f(__ldg(col + k));
+}
+
+template <int KIND>
+struct VertexK final : Vertex {
+  static constexpr int U = KIND == 0 ? 1 : KIND == 1 ? 1 : KIND == 2 ? 4 : 8;
+  __device__ explicit VertexK(const void* arg) : Vertex(arg) {}
+
+  __device__ void bfs_expand(vf_graph_bfs_args a) override {
+    const uint64_t b = a.offs_dev[vid];
+    for_neighbors<U>(a.col_dev, b, b + deg, [&](uint32_t u) {
+      if (a.depth_dev[u] == -1 && atomicCAS(a.depth_dev + u, -1, a.level + 1) == -1)
+        a.next_queue_dev[atomicAdd(a.next_count_dev, 1u)] = a.vobj_dev[u];
+    });
+  }
+  // bottom-up step: an unvisited vertex joins level+1 if a neighbour is at `level`
+  __device__ void bfs_probe(vf_graph_bfs_args a) override {
+    if (a.depth_dev[vid] != -1) return;
+    const uint64_t b = a.offs_dev[vid];
+    for (uint64_t k = b; k < b + deg; ++k) {
+      if (a.depth_dev[__ldg(a.col_dev + k)] == a.level) {
+        a.depth_dev[vid] = a.level + 1;
+        atomicAdd(a.next_count_dev, 1u);
+        return;
+      }
+    }
+  }
+  __device__ void cc_update(vf_graph_cc_args a) override {
+    const uint32_t own = a.label_in_dev[vid];
+    uint32_t m = own;
+    const uint64_t b = a.offs_dev[vid];
+    if constexpr (U == 1) {
+      for_neighbors<1>(a.col_dev, b, b + deg, [&](uint32_t u) { m = min(m, __ldg(a.label_in_dev + u)); });
+    } else {
+      uint32_t acc[U];
+#pragma unroll
+      for (int j = 0; j < U; ++j) acc[j] = own;
+      uint64_t k = b;
+      const uint64_t e = b + deg;
+      for (; k + U <= e; k += U) {
+#pragma unroll
+        for (int j = 0; j < U; ++j) acc[j] = min(acc[j], __ldg(a.label_in_dev + __ldg(a.col_dev + k + j)));
+      }
+      for (; k < e; ++k) acc[0] = min(acc[0], __ldg(a.label_in_dev + __ldg(a.col_dev + k)));
+#pragma unroll
+      for (int j = 0; j < U; ++j) m = min(m, acc[j]);
+    }
+    a.label_out_dev[vid] = m;
+    if (m != own) a.changed_dev[0] = 1u;
+  }
+  __device__ void pr_contrib(vf_graph_pr_args a) override {
+    const float r = a.rank_in_dev[vid];
+    a.contrib_dev[vid] = deg ? (double)r / (double)deg : 0.0;
+    if (!deg) atomicAdd(a.dangling_dev, (double)r);
+  }
+  __device__ void pr_update(vf_graph_pr_args a) override {
+    const uint64_t b = a.offs_dev[vid];
+    double s;
+    if constexpr (U == 1) {
+      s = 0.0;
+      for_neighbors<1>(a.col_dev, b, b + deg, [&](uint32_t u) { s += __ldg(a.contrib_dev + u); });
+    } else {
+      double acc[U];
+#pragma unroll
+      for (int j = 0; j < U; ++j) acc[j] = 0.0;
+      uint64_t k = b;
+      const uint64_t e = b + deg;
+      for (; k + U <= e; k += U) {
+#pragma unroll
+        for (int j = 0; j < U; ++j) acc[j] += __ldg(a.contrib_dev + __ldg(a.col_dev + k + j));
+      }
+      for (; k < e; ++k) acc[0] += __ldg(a.contrib_dev + __ldg(a.col_dev + k));
+      s = 0.0;
+#pragma unroll
+      for (int j = 0; j < U; ++j) s += acc[j];
+    }
+    const double D = *a.dangling_dev;
+    // (1-d)/V + d*(s + D/V), the oracle's operation order, IEEE fp64 (no contraction)
+    a.rank_out_dev[vid] = (float)__dadd_rn(a.base, __dmul_rn(a.d, __dadd_rn(s, __ddiv_rn(D, a.Vd))));
+  }
+};
+
+struct App {
+  static constexpr int kTypes = 4;
+  static constexpr int kMethods = 5;
+  static constexpr int kUnroll = 2;
+  static constexpr int kUnrollSorted = 2;
+  static constexpr int kPrefetch = 2;
+  using Base = Vertex;
+  template <int K>
+  using Type = VertexK<K>;
+
+  template <int M>
+  __device__ __forceinline__ static void vcall(Base* o, uint64_t, const ArgBlob& b) {
+    if constexpr (M == VF_GRAPH_BFS_EXPAND) o->bfs_expand(blob_as<vf_graph_bfs_args>(b));
+    else if constexpr (M == VF_GRAPH_BFS_PROBE) o->bfs_probe(blob_as<vf_graph_bfs_args>(b));
+    else if constexpr (M == VF_GRAPH_CC_UPDATE) o->cc_update(blob_as<vf_graph_cc_args>(b));
+    else if constexpr (M == VF_GRAPH_PR_CONTRIB) o->pr_contrib(blob_as<vf_graph_pr_args>(b));
+    else o->pr_update(blob_as<vf_graph_pr_args>(b));
+  }
+  template <int M, int K>
+  __device__ __forceinline__ static void dcall(Type<K>* o, uint64_t, const ArgBlob& b) {
+    if constexpr (M == VF_GRAPH_BFS_EXPAND) o->Type<K>::bfs_expand(blob_as<vf_graph_bfs_args>(b));
+    else if constexpr (M == VF_GRAPH_BFS_PROBE) o->Type<K>::bfs_probe(blob_as<vf_graph_bfs_args>(b));
+    else if constexpr (M == VF_GRAPH_CC_UPDATE) o->Type<K>::cc_update(blob_as<vf_graph_cc_args>(b));
+    else if constexpr (M == VF_GRAPH_PR_CONTRIB) o->Type<K>::pr_contrib(blob_as<vf_graph_pr_args>(b));
+    else o->Type<K>::pr_update(blob_as<vf_graph_pr_args>(b));
+  }
+  __device__ static void construct(uint32_t t, void* mem, const void* arg) {
+    construct_switch<App>(t, mem, arg);
+  }
+  __device__ static Base* make(uint32_t t, const void* arg) { return make_switch<App>(t, arg); }
+};
+static_assert(sizeof(VertexK<0>) == 16, "vertex layout");
+
+__global__ void k_bfs_init(uint64_t V, int32_t* depth, uint32_t src, const uint64_t* vobj, uint64_t* queue,
+                           uint32_t* count) {
+  const uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (v < V) depth[v] = v == src ? 0 : -1;
+  if (v == 0) {
+    queue[0] = vobj[src];
+    *count = 1;
+  }
+}
+
+__global__ void k_iota(uint64_t V, uint32_t* x) {
+  const uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (v < V) x[v] = (uint32_t)v;
+}
+
+__global__ void k_fill_f32(uint64_t V, float* x, float val) {
+  const uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (v < V) x[v] = val;
+}
+
+}  // namespace graph
+
+static const uint32_t kGraphBytes[4] = {16, 16, 16, 16};
+static const uint32_t kGraphArgs[5] = {sizeof(vf_graph_bfs_args), sizeof(vf_graph_bfs_args),
+                                       sizeof(vf_graph_cc_args), sizeof(vf_graph_pr_args),
+                                       sizeof(vf_graph_pr_args)};
+
+const AppOps* app_graph() {
+  static const AppOps ops = make_ops<graph::App>("graph", kGraphBytes, kGraphArgs);
+  return &ops;
+}
+
+}  // namespace vf
+
+extern "C" vf_status vf_graph_bfs_init(uint64_t V, int32_t* depth_dev, uint32_t src, const uint64_t* vobj_dev,
+                                       uint64_t* queue_dev, uint32_t* count_dev, void* stream) {
+  if (!V || src >= V || !depth_dev || !vobj_dev || !queue_dev || !count_dev) return VF_ERR_INVALID;
+  vf::graph::k_bfs_init<<<(unsigned)((V + 255) / 256), 256, 0, (cudaStream_t)stream>>>(V, depth_dev, src, vobj_dev,
+                                                                                       queue_dev, count_dev);
+  vf::note_launch();
+  return cudaGetLastError() == cudaSuccess ? VF_OK : VF_ERR_CUDA;
+}
+
+extern "C" vf_status vf_iota_u32(uint64_t n, uint32_t* x_dev, void* stream) {
+  if (!n) return VF_OK;
+  if (!x_dev) return VF_ERR_INVALID;
+  vf::graph::k_iota<<<(unsigned)((n + 255) / 256), 256, 0, (cudaStream_t)stream>>>(n, x_dev);
+  vf::note_launch();
+  return cudaGetLastError() == cudaSuccess ? VF_OK : VF_ERR_CUDA;
+}
+
+extern "C" vf_status vf_fill_f32(uint64_t n, float* x_dev, float value, void* stream) {
+  if (!n) return VF_OK;
+  if (!x_dev) return VF_ERR_INVALID;
+  vf::graph::k_fill_f32<<<(unsigned)((n + 255) / 256), 256, 0, (cudaStream_t)stream>>>(n, x_dev, value);
+  vf::note_launch();
+  return cudaGetLastError() == cudaSuccess ? VF_OK : VF_ERR_CUDA;
+}

@@ -36,6 +36,7 @@ static const AppOps* app_ops(uint32_t app) {
     case VF_APP_MICRO: return app_micro();
     case VF_APP_GOL: return app_gol();
     case VF_APP_GEN: return app_gen();
+    case VF_APP_GRAPH: return app_graph();
   }
   return nullptr;
 }

@@ -60,6 +60,7 @@ struct AppOps {
 const AppOps* app_micro();
 const AppOps* app_gol();
 const AppOps* app_gen();
+const AppOps* app_graph();
 
 // Benchmark / ablation knobs set through vf_set_tuning (-1 = app default).
 struct Tuning {

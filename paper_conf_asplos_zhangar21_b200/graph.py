@@ -1,0 +1,178 @@
+"""Config 4 driver: BFS / CC / PageRank over polymorphic vertices (Table 2).
+
+Argument marshalling and step sequencing over the C ABI only: vertex objects
+are allocated through libvf (typed arenas by degree bucket, or device-heap
+`new` for the CUDA baseline), and every per-vertex computation is a virtual
+method call dispatched by libvf (vf_dispatch). Host code reads back one scalar
+per BFS level / CC iteration to decide termination.
+
+Multi-GPU (``rank``/``world``): vertex ids are split into contiguous blocks;
+each rank dispatches only its owned vertices and the per-iteration state
+(depth / labels / contributions) is exchanged with an all-gather over the
+process group (NCCL on B200, gloo on CPU tests).
+"""
+from __future__ import annotations
+
+import ctypes
+
+import numpy as np
+import torch
+
+import synth
+
+from . import vf
+
+
+def _sync_scalar(t):
+    return int(t.item())
+
+
+class Graph:
+    def __init__(self, ctx: vf.Ctx, offs: np.ndarray, col: np.ndarray, variant: str = "typeptr",
+                 rank: int = 0, world: int = 1, group=None):
+        self.ctx, self.variant = ctx, variant
+        self.v = vf.VARIANTS[variant]
+        dev = torch.device(f"cuda:{ctx.device}")
+        self.dev = dev
+        V = len(offs) - 1
+        self.V = V
+        self.rank, self.world, self.group = rank, world, group
+        # owned vertex block [lo, hi)
+        per = (V + world - 1) // world
+        self.lo, self.hi = min(V, rank * per), min(V, (rank + 1) * per)
+        self.per = per
+        self.offs = torch.from_numpy(np.ascontiguousarray(offs, dtype=np.uint64).view(np.int64)).to(dev)
+        self.col = torch.from_numpy(np.ascontiguousarray(col, dtype=np.uint32).view(np.int32)).to(dev)
+        deg = np.diff(np.asarray(offs, dtype=np.int64))
+        types = synth.vertex_types(offs)
+        self.types_np = types
+        own = np.arange(self.lo, self.hi)
+        ctor = np.stack([own.astype(np.uint32), deg[own].astype(np.uint32)], axis=1).copy()
+        ctor_t = torch.from_numpy(ctor.view(np.int32)).to(dev)
+        tt = torch.from_numpy(types[own].astype(np.int32)).to(dev)
+        if variant == "cuda":
+            objs = ctx.alloc_cuda(vf.APP_GRAPH, tt, ctor_t)
+        else:
+            objs = ctx.alloc_typed_batch(vf.APP_GRAPH, tt, ctor_t, tag=(variant == "typeptr"))
+        # vobj is indexed by global vertex id; only the owned block is filled on this rank
+        self.vobj = torch.zeros(V, dtype=torch.int64, device=dev)
+        self.vobj[self.lo:self.hi] = objs
+        self.owned = self.vobj[self.lo:self.hi]
+        self.depth = torch.empty(V, dtype=torch.int32, device=dev)
+        self.q = [torch.empty(max(V, 1), dtype=torch.int64, device=dev) for _ in range(2)]
+        self.count = torch.zeros(1, dtype=torch.int32, device=dev)
+        self.lab = [torch.empty(V, dtype=torch.int32, device=dev) for _ in range(2)]
+        self.changed = torch.zeros(1, dtype=torch.int32, device=dev)
+        self.rk = [torch.empty(V, dtype=torch.float32, device=dev) for _ in range(2)]
+        self.contrib = torch.empty(V, dtype=torch.float64, device=dev)
+        self.dangling = torch.zeros(1, dtype=torch.float64, device=dev)
+        self.calls = 0
+        torch.cuda.synchronize(dev)
+
+    # ---------------------------------------------------------------- helpers
+    def _allgather_block(self, t):
+        """all-gather of the owned block of a per-vertex array (multi-GPU exchange, §8e)."""
+        if self.world == 1:
+            return
+        import torch.distributed as dist
+        padded = torch.zeros(self.per * self.world, dtype=t.dtype, device=t.device)
+        padded[:self.V] = t
+        out = list(padded.view(self.world, self.per).unbind(0))
+        dist.all_gather(out, padded[self.rank * self.per:(self.rank + 1) * self.per].clone(), group=self.group)
+        t.copy_(torch.stack(out).view(-1)[:self.V])
+
+    def _allreduce_sum(self, t):
+        if self.world == 1:
+            return
+        import torch.distributed as dist
+        dist.all_reduce(t, group=self.group)
+
+    def _dispatch(self, method, objs_ptr, n, args, stream=None):
+        st = self.ctx.dispatch_raw(self.v, vf.APP_GRAPH, method, objs_ptr, n, args, vf._stream(stream))
+        if st:
+            self.ctx._check(st, f"graph method {method}")
+
+    # ---------------------------------------------------------------- BFS
+    def bfs(self, src: int, mode: str = "topdown"):
+        """Level-synchronous BFS from src; returns (depth tensor, levels, calls).
+        topdown: one virtual bfs_expand() per frontier vertex (single GPU);
+        bottomup: one virtual bfs_probe() per owned vertex per level (multi-GPU)."""
+        L = vf.lib()
+        st = L.vf_graph_bfs_init(self.V, self.depth.data_ptr(), src, self.vobj.data_ptr(), self.q[0].data_ptr(),
+                                 self.count.data_ptr(), vf._stream(None))
+        if st:
+            raise vf.VFError(st, "bfs_init")
+        calls, level = 0, 0
+        if mode == "topdown" and self.world == 1:
+            n = 1
+            while n > 0:
+                self.count.zero_()
+                a = vf.graph_bfs_args(self.offs.data_ptr(), self.col.data_ptr(), self.depth.data_ptr(),
+                                      self.vobj.data_ptr(), self.q[1].data_ptr(), self.count.data_ptr(), level)
+                self._dispatch(vf.GRAPH_BFS_EXPAND, self.q[0].data_ptr(), n, a)
+                calls += n
+                n = _sync_scalar(self.count)
+                self.q[0], self.q[1] = self.q[1], self.q[0]
+                level += 1
+        else:
+            nown = self.hi - self.lo
+            while True:
+                self.count.zero_()
+                a = vf.graph_bfs_args(self.offs.data_ptr(), self.col.data_ptr(), self.depth.data_ptr(),
+                                      self.vobj.data_ptr(), 0, self.count.data_ptr(), level)
+                self._dispatch(vf.GRAPH_BFS_PROBE, self.owned.data_ptr(), nown, a)
+                calls += nown
+                self._allreduce_sum(self.count)
+                self._allgather_block(self.depth)
+                level += 1
+                if _sync_scalar(self.count) == 0:
+                    break
+        self.calls = calls
+        return self.depth, level, calls
+
+    # ---------------------------------------------------------------- CC
+    def cc(self, max_iters: int = 10 ** 6):
+        """Jacobi min-label propagation until no label changes; returns (labels, iters, calls)."""
+        L = vf.lib()
+        L.vf_iota_u32(self.V, self.lab[0].data_ptr(), vf._stream(None))
+        it, calls, nown = 0, 0, self.hi - self.lo
+        while it < max_iters:
+            self.changed.zero_()
+            a = vf.graph_cc_args(self.offs.data_ptr(), self.col.data_ptr(), self.lab[0].data_ptr(),
+                                 self.lab[1].data_ptr(), self.changed.data_ptr())
+            self._dispatch(vf.GRAPH_CC_UPDATE, self.owned.data_ptr(), nown, a)
+            calls += nown
+            it += 1
+            self._allgather_block(self.lab[1])
+            self._allreduce_sum(self.changed)
+            self.lab[0], self.lab[1] = self.lab[1], self.lab[0]
+            if _sync_scalar(self.changed) == 0:
+                break
+        self.calls = calls
+        return self.lab[0], it, calls
+
+    # ---------------------------------------------------------------- PageRank
+    def pr_init(self):
+        vf.lib().vf_fill_f32(self.V, self.rk[0].data_ptr(), ctypes.c_float(1.0 / self.V).value, vf._stream(None))
+
+    def pr_iteration(self, d: float = 0.85, stream=None):
+        """One PageRank iteration = virtual pr_contrib() + pr_update() per owned vertex."""
+        nown = self.hi - self.lo
+        self.dangling.zero_()
+        a = vf.graph_pr_args(self.offs.data_ptr(), self.col.data_ptr(), self.rk[0].data_ptr(), self.rk[1].data_ptr(),
+                             self.contrib.data_ptr(), self.dangling.data_ptr(), (1.0 - d) / self.V, d, float(self.V))
+        self._dispatch(vf.GRAPH_PR_CONTRIB, self.owned.data_ptr(), nown, a, stream)
+        self._allgather_block(self.contrib)
+        self._allreduce_sum(self.dangling)
+        self._dispatch(vf.GRAPH_PR_UPDATE, self.owned.data_ptr(), nown, a, stream)
+        self._allgather_block(self.rk[1])
+        self.rk[0], self.rk[1] = self.rk[1], self.rk[0]
+        return 2 * nown
+
+    def pagerank(self, iters: int = 20, d: float = 0.85):
+        self.pr_init()
+        calls = 0
+        for _ in range(iters):
+            calls += self.pr_iteration(d)
+        self.calls = calls
+        return self.rk[0], calls

@@ -19,10 +19,11 @@ SO = os.path.join(PKG, "libvf.so")
 VF_OK = 0
 CUDA, SHAREDOA, COAL, TYPEPTR = 0, 1, 2, 3
 VARIANTS = {"cuda": CUDA, "sharedoa": SHAREDOA, "coal": COAL, "typeptr": TYPEPTR}
-APP_MICRO, APP_GOL, APP_GEN = 0, 1, 2
+APP_MICRO, APP_GOL, APP_GEN, APP_GRAPH = 0, 1, 2, 3
 MICRO_APPLY, MICRO_GET = 0, 1
 GOL_NEXT, GOL_GET = 0, 1
 GEN_NEXT, GEN_GET = 0, 1
+GRAPH_BFS_EXPAND, GRAPH_BFS_PROBE, GRAPH_CC_UPDATE, GRAPH_PR_CONTRIB, GRAPH_PR_UPDATE = 0, 1, 2, 3, 4
 NOT_FOUND = 0xFFFFFFFF
 VA_BITS = 57
 MAX_RANGES = 4096
@@ -37,6 +38,7 @@ SYMBOLS = [
     "vf_regions", "vf_type_vptrs", "vf_resolve", "vf_verify_types", "vf_dispatch_cuda",
     "vf_dispatch_sharedoa", "vf_dispatch_coal", "vf_dispatch_typeptr", "vf_dispatch",
     "vf_gol_neighbors", "vf_gol_swap", "vf_gen_swap", "vf_checksum_i32", "vf_launch_count", "vf_set_tuning",
+    "vf_graph_bfs_init", "vf_iota_u32", "vf_fill_f32",
 ]
 
 
@@ -83,6 +85,24 @@ class gen_next_args(ctypes.Structure):
 gen_get_args = gol_get_args
 
 
+class graph_bfs_args(ctypes.Structure):
+    _fields_ = [("offs_dev", ctypes.c_void_p), ("col_dev", ctypes.c_void_p), ("depth_dev", ctypes.c_void_p),
+                ("vobj_dev", ctypes.c_void_p), ("next_queue_dev", ctypes.c_void_p),
+                ("next_count_dev", ctypes.c_void_p), ("level", ctypes.c_int32)]
+
+
+class graph_cc_args(ctypes.Structure):
+    _fields_ = [("offs_dev", ctypes.c_void_p), ("col_dev", ctypes.c_void_p), ("label_in_dev", ctypes.c_void_p),
+                ("label_out_dev", ctypes.c_void_p), ("changed_dev", ctypes.c_void_p)]
+
+
+class graph_pr_args(ctypes.Structure):
+    _fields_ = [("offs_dev", ctypes.c_void_p), ("col_dev", ctypes.c_void_p), ("rank_in_dev", ctypes.c_void_p),
+                ("rank_out_dev", ctypes.c_void_p), ("contrib_dev", ctypes.c_void_p),
+                ("dangling_dev", ctypes.c_void_p), ("base", ctypes.c_double), ("d", ctypes.c_double),
+                ("Vd", ctypes.c_double)]
+
+
 _lib = None
 
 
@@ -122,6 +142,9 @@ def lib(required: bool = True):
         "vf_checksum_i32": (I, [P, U64, P, P]),
         "vf_launch_count": (U64, []),
         "vf_set_tuning": (I, [ctypes.c_char_p, I]),
+        "vf_graph_bfs_init": (I, [U64, P, U32, P, P, P, P]),
+        "vf_iota_u32": (I, [U64, P, P]),
+        "vf_fill_f32": (I, [U64, P, ctypes.c_float, P]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)
