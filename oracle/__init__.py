@@ -27,7 +27,7 @@ import numpy as np
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 SO = os.path.join(HERE, "liboracle.so")
-SOURCES = ["alloc.cpp", "micro.cpp", "gol.cpp", "gen.cpp", "graph.cpp"]
+SOURCES = ["alloc.cpp", "micro.cpp", "gol.cpp", "gen.cpp", "graph.cpp", "ray.cpp"]
 NOT_FOUND = 0xFFFFFFFF
 
 
@@ -89,6 +89,9 @@ def lib():
         L.oracle_graph_pr.restype = ctypes.c_int
         L.oracle_graph_pr.argtypes = [U64, P, P, P, ctypes.c_double, U32, ctypes.c_int, P,
                                       ctypes.POINTER(ctypes.c_double)]
+        L.oracle_ray_render.restype = ctypes.c_int
+        L.oracle_ray_render.argtypes = [U32, U32, U32, U32, U32, P, P, P, P, ctypes.c_int, P, P, P,
+                                        ctypes.POINTER(ctypes.c_double)]
         L.oracle_max_threads.restype = ctypes.c_int
         _lib = L
     return _lib
@@ -246,3 +249,22 @@ def graph_pr(offs, col, types, iters: int = 20, d: float = 0.85, threads: int = 
     if rc:
         raise ValueError(f"oracle_graph_pr rc={rc}")
     return rank, sec.value
+
+
+def ray_render(W: int, H: int, types, params, cam, albedo, row0: int = 0, nrows: int | None = None,
+               threads: int = 1):
+    """Returns (rgb float32[nrows, W, 3], hit_id int32[nrows, W], calls, seconds)."""
+    nrows = H - row0 if nrows is None else nrows
+    types = np.ascontiguousarray(types, dtype=np.uint32)
+    params = np.ascontiguousarray(params, dtype=np.float32)
+    cam = np.ascontiguousarray(cam, dtype=np.float32)
+    albedo = np.ascontiguousarray(albedo, dtype=np.float32)
+    rgb = np.zeros((nrows, W, 3), np.float32)
+    hid = np.zeros((nrows, W), np.int32)
+    calls, sec = ctypes.c_uint64(), ctypes.c_double()
+    rc = lib().oracle_ray_render(W, H, row0, nrows, len(types), types.ctypes.data, params.ctypes.data,
+                                 cam.ctypes.data, albedo.ctypes.data, threads, rgb.ctypes.data, hid.ctypes.data,
+                                 ctypes.byref(calls), ctypes.byref(sec))
+    if rc:
+        raise ValueError(f"oracle_ray_render rc={rc}")
+    return rgb, hid, calls.value, sec.value

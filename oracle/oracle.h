@@ -122,6 +122,19 @@ int oracle_graph_cc(uint64_t V, const uint64_t* offs, const uint32_t* col, const
 int oracle_graph_pr(uint64_t V, const uint64_t* offs, const uint32_t* col, const uint32_t* types,
                     double d, uint32_t iters, int threads, float* rank, double* seconds);
 
+/* ---- Config 3 ray tracer over polymorphic shapes (Table 2 RAY P:1592-1600;
+ * readings G24, G25). Shapes j = 0..S-1 of type types[j] (0 Plane y=h,
+ * 1 Sphere, 2 axis-aligned Rect, 3 Triangle) with 12 fp32 params each
+ * (params + 12 j). Rows [row0, row0+nrows) of a W x H image; per pixel one
+ * primary ray, one virtual hit() per shape in ascending id, closest t > 1e-4
+ * with strict '<' (ties -> smaller id), then one virtual normal() on the
+ * winner; rgb = fmaf(albedo[kind], max(0, n.l), 0.1), black and id -1 on a
+ * miss. cam = {tan(fov/2)*W/H, tan(fov/2), lx, ly, lz}. *calls = nrows*W*S. */
+int oracle_ray_render(uint32_t W, uint32_t H, uint32_t row0, uint32_t nrows, uint32_t S,
+                      const uint32_t* types, const float* params, const float* cam,
+                      const float* albedo, int threads, float* rgb, int32_t* hit_id,
+                      uint64_t* calls, double* seconds);
+
 /* number of OpenMP threads actually available */
 int oracle_max_threads(void);
 

@@ -197,6 +197,63 @@ def csr_from_edges(V: int, edges):
     return offs, col[:arcs].copy()
 
 
+# --------------------------------------------------------------------------
+# Config 3: ray-tracer scene (reading G24)
+# --------------------------------------------------------------------------
+RAY_ALBEDO = np.array([[0.8, 0.8, 0.8], [0.9, 0.2, 0.2], [0.2, 0.9, 0.2], [0.2, 0.3, 0.9]], np.float32)
+
+
+def _unit(seed, stream, idx):
+    """uniform float32 in [0, 1) with 24 random bits (exact)."""
+    return ((draw(seed, stream, idx) >> np.uint64(40)).astype(np.float32) * np.float32(2.0 ** -24))
+
+
+def ray_scene(S: int, seed: int = 7, ground: bool = True):
+    """Shapes j = 0..S-1: j = 0 is the ground plane y = -2 (if ground), else type
+    1 + (j mod 3) (Sphere, Rect, Triangle); centres uniform in
+    [-50,50]x[-30,30]x[-150,-50], sizes uniform in [0.5, 2). Returns
+    (types uint32[S], params float32[S, 12])."""
+    j = np.arange(S, dtype=np.uint64)
+    r = [_unit(seed, S_SCENE, j * np.uint64(16) + np.uint64(k)) for k in range(16)]
+    lo = np.array([-50, -30, -150], np.float32)
+    hi = np.array([50, 30, -50], np.float32)
+    c = np.stack([lo[k] + r[k] * (hi[k] - lo[k]) for k in range(3)], axis=1).astype(np.float32)
+    s = (np.float32(0.5) + r[3] * np.float32(1.5)).astype(np.float32)
+    types = (1 + (j % np.uint64(3))).astype(np.uint32)
+    P = np.zeros((S, 12), np.float32)
+    sph = types == 1
+    P[sph, 0:3] = c[sph]
+    P[sph, 3] = s[sph]
+    rect = types == 2
+    axis = np.minimum((r[4] * 3).astype(np.int64), 2)
+    for a in range(3):
+        m = rect & (axis == a)
+        oth = [k for k in range(3) if k != a]
+        P[m, 0] = a
+        P[m, 1] = c[m, a]
+        P[m, 2] = c[m, oth[0]] - s[m]
+        P[m, 3] = c[m, oth[0]] + s[m]
+        P[m, 4] = c[m, oth[1]] - s[m]
+        P[m, 5] = c[m, oth[1]] + s[m]
+    tri = types == 3
+    for v in range(3):
+        for k in range(3):
+            P[tri, 3 * v + k] = c[tri, k] + s[tri] * (np.float32(2.0) * r[5 + 3 * v + k][tri] - np.float32(1.0))
+    if ground and S > 0:
+        types[0] = 0
+        P[0, :] = 0
+        P[0, 0] = -2.0
+    return types, P
+
+
+def ray_camera(W: int, H: int, fov_deg: float = 60.0, light=(0.4, 1.0, 0.6)):
+    """fp32 camera constants computed once on the host: [tan(fov/2)*W/H, tan(fov/2), unit light]."""
+    th = np.tan(np.deg2rad(fov_deg) / 2.0)
+    l = np.asarray(light, np.float64)
+    l = l / np.linalg.norm(l)
+    return np.array([th * W / H, th, l[0], l[1], l[2]], np.float32)
+
+
 # degree-bucket vertex types (SURVEY W6, reading G22): Leaf <=1, Low 2-15, Mid 16-255, Hub >=256
 DEG_BOUNDS = (1, 15, 255)
 
