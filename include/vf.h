@@ -65,7 +65,8 @@ enum {
   VF_APP_GOL = 1,   /* config 1: Cell / Alive / Dead               (Table 2)  */
   VF_APP_GEN = 2,   /* config 5: Cell / Dead / Alive / Dying       (Table 2)  */
   VF_APP_GRAPH = 3, /* config 4: Vertex / Leaf / Low / Mid / Hub   (Table 2)  */
-  VF_APP_COUNT = 4
+  VF_APP_RAY = 4,   /* config 3: Shape / Plane / Sphere / Rect / Triangle   */
+  VF_APP_COUNT = 5
 };
 
 /* Methods of VF_APP_MICRO (args structs are passed by value, see dispatch). */
@@ -271,6 +272,20 @@ vf_status vf_gol_swap(vf_ctx* ctx, uint64_t ncells, const uint8_t* state_prev_de
 vf_status vf_gen_swap(vf_ctx* ctx, uint64_t ncells, const uint8_t* state_prev_dev,
                       const uint8_t* state_next_dev, uint64_t* grid_dev, const uint64_t* dead_dev,
                       const uint64_t* alive_dev, const uint64_t* dying_dev, void* stream);
+
+/* Config 3 ray tracer (readings G24, G25): render rows [row0, row0+nrows) of
+ * a W x H image over S shapes of VF_APP_RAY (type ids 0 Plane, 1 Sphere,
+ * 2 Rect, 3 Triangle; constructor argument = 12 fp32 params, see
+ * synth.ray_scene). Per pixel: one primary ray through the pixel centre, one
+ * virtual hit() per shape in ascending id (CUDA / SHAREDOA: virtual call;
+ * COAL / TYPEPTR: type from the pointer, direct inlined call), closest
+ * t > 1e-4 with ties to the smaller id, Lambert shading with 0.1 ambient.
+ * cam (host, 5 floats) = {tan(fov/2)*W/H, tan(fov/2), unit light xyz};
+ * albedo (host, 12 floats) = rgb per type. Writes rgb_dev[nrows*W*3] (fp32)
+ * and hit_dev[nrows*W] (shape id or -1). Bit-identical to the CPU oracle. */
+vf_status vf_ray_render(vf_ctx* ctx, vf_variant v, const uint64_t* shapes_dev, uint32_t S, uint32_t W,
+                        uint32_t H, uint32_t row0, uint32_t nrows, const float* cam, const float* albedo,
+                        float* rgb_dev, int32_t* hit_dev, void* stream);
 
 /* Graph helpers: BFS start state (depth = -1 except depth[src] = 0, queue =
  * [vobj[src]], *count = 1), iota (x[i] = i), fill (x[i] = value). */

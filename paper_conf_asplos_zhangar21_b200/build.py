@@ -28,8 +28,15 @@ def _headers():
         [os.path.join(ROOT, "include", "vf.h")]
 
 
+# Float apps whose results must match the CPU oracle bit for bit: no FMA
+# contraction (every FMA is an explicit fmaf in the source), IEEE div/sqrt.
+PER_FILE = {"app_ray.cu": ["-fmad=false", "-prec-div=true", "-prec-sqrt=true", "-ftz=false"],
+            "app_nbody.cu": ["-fmad=false", "-prec-div=true", "-prec-sqrt=true", "-ftz=false"],
+            "app_stut.cu": ["-fmad=false", "-prec-div=true", "-prec-sqrt=true", "-ftz=false"]}
+
+
 def _compile(src: str, obj: str, verbose: bool) -> str:
-    cmd = ["nvcc"] + FLAGS + ["-c", src, "-o", obj]
+    cmd = ["nvcc"] + FLAGS + PER_FILE.get(os.path.basename(src), []) + ["-c", src, "-o", obj]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         raise RuntimeError(f"nvcc failed for {src}:\n{r.stderr}")

@@ -37,6 +37,7 @@ static const AppOps* app_ops(uint32_t app) {
     case VF_APP_GOL: return app_gol();
     case VF_APP_GEN: return app_gen();
     case VF_APP_GRAPH: return app_graph();
+    case VF_APP_RAY: return app_ray();
   }
   return nullptr;
 }
@@ -704,6 +705,22 @@ vf_status vf_dispatch(vf_ctx* c, vf_variant v, uint32_t app, uint32_t method,
   memset(&blob, 0, sizeof blob);
   if (args_bytes) memcpy(blob.b, args, args_bytes);
   CUDA_TRY(c, ops->dispatch((int)v, method, objs_dev, n, blob, dev_table(c, app), S(stream)));
+  return VF_OK;
+}
+
+vf_status vf_ray_render(vf_ctx* c, vf_variant v, const uint64_t* shapes_dev, uint32_t S, uint32_t W,
+                        uint32_t H, uint32_t row0, uint32_t nrows, const float* cam, const float* albedo,
+                        float* rgb_dev, int32_t* hit_dev, void* stream) {
+  vf_status st = check_app(c, VF_APP_RAY);
+  if (st) return st;
+  if ((unsigned)v > VF_TYPEPTR) return fail(c, VF_ERR_INVALID, "variant %d", (int)v);
+  if (!cam || !albedo || !rgb_dev || !hit_dev || (S && !shapes_dev) || row0 + nrows > H)
+    return fail(c, VF_ERR_INVALID, "ray_render arguments");
+  if ((st = set_device(c)) || (st = ensure_vptrs(c, VF_APP_RAY))) return st;
+  if (v == VF_COAL && c->tables[VF_APP_RAY].K > VF_MAX_RANGES)
+    return fail(c, VF_ERR_TABLE_FULL, "K = %u > %u", c->tables[VF_APP_RAY].K, VF_MAX_RANGES);
+  CUDA_TRY(c, ray_render((int)v, shapes_dev, S, W, H, row0, nrows, cam, albedo, rgb_dev, hit_dev,
+                         dev_table(c, VF_APP_RAY), reinterpret_cast<cudaStream_t>(stream)));
   return VF_OK;
 }
 

@@ -61,6 +61,12 @@ const AppOps* app_micro();
 const AppOps* app_gol();
 const AppOps* app_gen();
 const AppOps* app_graph();
+const AppOps* app_ray();
+
+// config 3 renderer (app_ray.cu): rows [row0, row0+nrows) of a W x H image
+cudaError_t ray_render(int variant, const uint64_t* objs, uint32_t S, uint32_t W, uint32_t H, uint32_t row0,
+                       uint32_t nrows, const float* cam5, const float* albedo12, float* rgb, int32_t* hid,
+                       const DevTable& tbl, cudaStream_t s);
 
 // Benchmark / ablation knobs set through vf_set_tuning (-1 = app default).
 struct Tuning {

@@ -38,8 +38,9 @@ SYMBOLS = [
     "vf_regions", "vf_type_vptrs", "vf_resolve", "vf_verify_types", "vf_dispatch_cuda",
     "vf_dispatch_sharedoa", "vf_dispatch_coal", "vf_dispatch_typeptr", "vf_dispatch",
     "vf_gol_neighbors", "vf_gol_swap", "vf_gen_swap", "vf_checksum_i32", "vf_launch_count", "vf_set_tuning",
-    "vf_graph_bfs_init", "vf_iota_u32", "vf_fill_f32",
+    "vf_graph_bfs_init", "vf_iota_u32", "vf_fill_f32", "vf_ray_render",
 ]
+APP_RAY = 4
 
 
 class VFError(RuntimeError):
@@ -145,6 +146,7 @@ def lib(required: bool = True):
         "vf_graph_bfs_init": (I, [U64, P, U32, P, P, P, P]),
         "vf_iota_u32": (I, [U64, P, P]),
         "vf_fill_f32": (I, [U64, P, ctypes.c_float, P]),
+        "vf_ray_render": (I, [P, I, P, U32, U32, U32, U32, U32, P, P, P, P, P]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)
