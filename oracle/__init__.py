@@ -27,7 +27,7 @@ import numpy as np
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 SO = os.path.join(HERE, "liboracle.so")
-SOURCES = ["alloc.cpp", "micro.cpp", "gol.cpp", "gen.cpp", "graph.cpp", "ray.cpp"]
+SOURCES = ["alloc.cpp", "micro.cpp", "gol.cpp", "gen.cpp", "graph.cpp", "ray.cpp", "traf.cpp"]
 NOT_FOUND = 0xFFFFFFFF
 
 
@@ -92,6 +92,9 @@ def lib():
         L.oracle_ray_render.restype = ctypes.c_int
         L.oracle_ray_render.argtypes = [U32, U32, U32, U32, U32, P, P, P, P, ctypes.c_int, P, P, P,
                                         ctypes.POINTER(ctypes.c_double)]
+        L.oracle_traf_run.restype = ctypes.c_int
+        L.oracle_traf_run.argtypes = [U32, U32, U32, P, P, P, P, P, U32, U64, P, P, ctypes.c_int, P, P,
+                                      ctypes.POINTER(ctypes.c_double)]
         L.oracle_max_threads.restype = ctypes.c_int
         _lib = L
     return _lib
@@ -268,3 +271,19 @@ def ray_render(W: int, H: int, types, params, cam, albedo, row0: int = 0, nrows:
     if rc:
         raise ValueError(f"oracle_ray_render rc={rc}")
     return rgb, hid, calls.value, sec.value
+
+
+def traf_run(world: dict, steps: int, threads: int = 1):
+    """world = synth.traf_world(...); returns (pos uint32[nveh], v uint32[nveh], seconds)."""
+    w = {k: (np.ascontiguousarray(v) if isinstance(v, np.ndarray) else v) for k, v in world.items()}
+    n = len(w["veh_ring"])
+    pos = np.zeros(n, np.uint32)
+    vel = np.zeros(n, np.uint32)
+    sec = ctypes.c_double()
+    rc = lib().oracle_traf_run(w["R"], w["L"], n, w["veh_ring"].ctypes.data, w["veh_pos"].ctypes.data,
+                               w["veh_type"].ctypes.data, w["light"].ctypes.data, w["phase"].ctypes.data, steps,
+                               w["seed"], w["vmax"].ctypes.data, w["slow_thr"].ctypes.data, threads,
+                               pos.ctypes.data, vel.ctypes.data, ctypes.byref(sec))
+    if rc:
+        raise ValueError(f"oracle_traf_run rc={rc}")
+    return pos, vel, sec.value

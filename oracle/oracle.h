@@ -135,6 +135,21 @@ int oracle_ray_render(uint32_t W, uint32_t H, uint32_t row0, uint32_t nrows, uin
                       const float* albedo, int threads, float* rgb, int32_t* hit_id,
                       uint64_t* calls, double* seconds);
 
+/* ---- Config 5 TRAF: Nagel-Schreckenberg rings (Table 2 P:1513-1516;
+ * reading G16). R rings x L cells; cell c (global ring*L + pos) is a
+ * LightCell if light[c] (phase[c]) else a PlainCell; vehicle i of type
+ * veh_type[i] (0 Car, 1 Truck, 2 Bus; vmax[], slow_thr[] per type) starts at
+ * (veh_ring[i], veh_pos[i]) with v = 0. Per step t: virtual update(t) per
+ * cell (blocked = light red: (t+phase) mod 20 < 8), then virtual step() per
+ * vehicle against the previous occupancy (see traf.cpp), occupancy rebuilt.
+ * Writes final pos_out / v_out per vehicle. Returns 2 if two vehicles share
+ * a starting cell. */
+int oracle_traf_run(uint32_t R, uint32_t L, uint32_t nveh, const uint32_t* veh_ring,
+                    const uint32_t* veh_pos, const uint32_t* veh_type, const uint8_t* light,
+                    const uint32_t* phase, uint32_t steps, uint64_t seed, const uint32_t* vmax,
+                    const uint32_t* slow_thr, int threads, uint32_t* pos_out, uint32_t* v_out,
+                    double* seconds);
+
 /* number of OpenMP threads actually available */
 int oracle_max_threads(void);
 

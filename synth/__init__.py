@@ -254,6 +254,33 @@ def ray_camera(W: int, H: int, fov_deg: float = 60.0, light=(0.4, 1.0, 0.6)):
     return np.array([th * W / H, th, l[0], l[1], l[2]], np.float32)
 
 
+# --------------------------------------------------------------------------
+# Config 5 TRAF: Nagel-Schreckenberg rings (reading G16)
+# --------------------------------------------------------------------------
+TRAF_VMAX = np.array([5, 3, 4], np.uint32)          # Car, Truck, Bus
+TRAF_PSLOW = (0.2, 0.1, 0.3)
+
+
+def traf_world(R: int, L: int, density: float = 0.25, light_p: float = 1.0 / 32, seed: int = 11,
+               p_slow=TRAF_PSLOW):
+    """Rings x cells world: vehicles on cells with Bernoulli(density) draws (ring-major
+    id order), type uniform in {Car, Truck, Bus}; LightCells with Bernoulli(light_p),
+    phase uniform in [0, 20)."""
+    N = R * L
+    c = np.arange(N, dtype=np.uint64)
+    occ = bernoulli(draw(seed, S_TRAF, c), density)
+    cells = np.nonzero(occ)[0]
+    veh_ring = (cells // L).astype(np.uint32)
+    veh_pos = (cells % L).astype(np.uint32)
+    vid = np.arange(len(cells), dtype=np.uint64)
+    veh_type = uniform(draw(seed, S_TRAF, vid + np.uint64(1 << 40)), 3)
+    light = bernoulli(draw(seed, S_TRAF, c + np.uint64(1 << 41)), light_p).astype(np.uint8)
+    phase = uniform(draw(seed, S_TRAF, c + np.uint64(1 << 42)), 20)
+    slow_thr = np.array([int(p * (1 << 32)) for p in p_slow], np.uint32)
+    return dict(R=R, L=L, veh_ring=veh_ring, veh_pos=veh_pos, veh_type=veh_type, light=light, phase=phase,
+                seed=seed, vmax=TRAF_VMAX.copy(), slow_thr=slow_thr)
+
+
 # degree-bucket vertex types (SURVEY W6, reading G22): Leaf <=1, Low 2-15, Mid 16-255, Hub >=256
 DEG_BOUNDS = (1, 15, 255)
 
