@@ -66,8 +66,41 @@ enum {
   VF_APP_GEN = 2,   /* config 5: Cell / Dead / Alive / Dying       (Table 2)  */
   VF_APP_GRAPH = 3, /* config 4: Vertex / Leaf / Low / Mid / Hub   (Table 2)  */
   VF_APP_RAY = 4,   /* config 3: Shape / Plane / Sphere / Rect / Triangle   */
-  VF_APP_COUNT = 5
+  VF_APP_TRAF = 5,  /* config 5: Agent / PlainCell / LightCell / Car / Truck / Bus        */
+  VF_APP_COUNT = 6
 };
+
+/* Methods of VF_APP_TRAF (Table 2, reading G16). Type ids: 0
+ * PlainCell, 1 LightCell (ctor arg {u32 cell, u32 phase}); 2 Car, 3 Truck,
+ * 4 Bus (ctor arg {u32 id, u32 ring, u32 pos, u32 pad}). Cells are indexed
+ * globally (ring * L + pos). */
+enum {
+  VF_TRAF_CELL_UPDATE = 0, /* blocked[c] = LightCell red ((t+phase) mod 20 < 8); occ_next[c] = 0 */
+  VF_TRAF_VEH_STEP = 1,    /* Nagel-Schreckenberg step against occ / blocked; sets occ_next  */
+  VF_TRAF_GET = 2,         /* pos_out[id], v_out[id]                                          */
+  VF_TRAF_PLACE = 3        /* occ[ring*L + pos] = 1 (initial occupancy)                        */
+};
+typedef struct {
+  uint8_t* blocked_dev;
+  uint8_t* occ_next_dev;
+  uint32_t t;
+} vf_traf_cell_args;
+typedef struct {
+  const uint8_t* occ_dev;
+  const uint8_t* blocked_dev;
+  uint8_t* occ_next_dev;
+  uint32_t L, t;
+  uint64_t seed;
+  uint32_t vmax[3];
+  uint32_t slow_thr[3];
+} vf_traf_step_args;
+typedef struct {
+  uint32_t* pos_out_dev;  /* indexed by id - id_base (vehicle ids are global, ring-major) */
+  uint32_t* v_out_dev;
+  uint8_t* occ_dev;
+  uint32_t L;
+  uint32_t id_base;
+} vf_traf_get_args;
 
 /* Methods of VF_APP_MICRO (args structs are passed by value, see dispatch). */
 enum { VF_MICRO_APPLY = 0, /* args: none                                       */

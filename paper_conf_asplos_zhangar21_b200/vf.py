@@ -41,6 +41,23 @@ SYMBOLS = [
     "vf_graph_bfs_init", "vf_iota_u32", "vf_fill_f32", "vf_ray_render",
 ]
 APP_RAY = 4
+APP_TRAF = 5
+TRAF_CELL_UPDATE, TRAF_VEH_STEP, TRAF_GET, TRAF_PLACE = 0, 1, 2, 3
+
+
+class traf_cell_args(ctypes.Structure):
+    _fields_ = [("blocked_dev", ctypes.c_void_p), ("occ_next_dev", ctypes.c_void_p), ("t", ctypes.c_uint32)]
+
+
+class traf_step_args(ctypes.Structure):
+    _fields_ = [("occ_dev", ctypes.c_void_p), ("blocked_dev", ctypes.c_void_p), ("occ_next_dev", ctypes.c_void_p),
+                ("L", ctypes.c_uint32), ("t", ctypes.c_uint32), ("seed", ctypes.c_uint64),
+                ("vmax", ctypes.c_uint32 * 3), ("slow_thr", ctypes.c_uint32 * 3)]
+
+
+class traf_get_args(ctypes.Structure):
+    _fields_ = [("pos_out_dev", ctypes.c_void_p), ("v_out_dev", ctypes.c_void_p), ("occ_dev", ctypes.c_void_p),
+                ("L", ctypes.c_uint32), ("id_base", ctypes.c_uint32)]
 
 
 class VFError(RuntimeError):
