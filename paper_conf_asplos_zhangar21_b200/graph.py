@@ -27,6 +27,32 @@ def _sync_scalar(t):
     return int(t.item())
 
 
+def block_range(V: int, rank: int, world: int):
+    """Owned vertex block [lo, hi) of `rank` and the per-rank block size."""
+    per = (V + world - 1) // world
+    return min(V, rank * per), min(V, (rank + 1) * per), per
+
+
+def allgather_block(t, V: int, per: int, rank: int, world: int, group=None):
+    """In-place all-gather of each rank's owned block of a per-vertex array (§8e):
+    after the call every rank holds every rank's block."""
+    if world == 1:
+        return
+    import torch.distributed as dist
+    padded = torch.zeros(per * world, dtype=t.dtype, device=t.device)
+    padded[:V] = t
+    out = [torch.empty(per, dtype=t.dtype, device=t.device) for _ in range(world)]
+    dist.all_gather(out, padded[rank * per:(rank + 1) * per].clone(), group=group)
+    t.copy_(torch.cat(out)[:V])
+
+
+def allreduce_sum(t, world: int, group=None):
+    if world == 1:
+        return
+    import torch.distributed as dist
+    dist.all_reduce(t, group=group)
+
+
 class Graph:
     def __init__(self, ctx: vf.Ctx, offs: np.ndarray, col: np.ndarray, variant: str = "typeptr",
                  rank: int = 0, world: int = 1, group=None):
@@ -38,9 +64,7 @@ class Graph:
         self.V = V
         self.rank, self.world, self.group = rank, world, group
         # owned vertex block [lo, hi)
-        per = (V + world - 1) // world
-        self.lo, self.hi = min(V, rank * per), min(V, (rank + 1) * per)
-        self.per = per
+        self.lo, self.hi, self.per = block_range(V, rank, world)
         self.offs = torch.from_numpy(np.ascontiguousarray(offs, dtype=np.uint64).view(np.int64)).to(dev)
         self.col = torch.from_numpy(np.ascontiguousarray(col, dtype=np.uint32).view(np.int32)).to(dev)
         deg = np.diff(np.asarray(offs, dtype=np.int64))
@@ -71,21 +95,10 @@ class Graph:
 
     # ---------------------------------------------------------------- helpers
     def _allgather_block(self, t):
-        """all-gather of the owned block of a per-vertex array (multi-GPU exchange, §8e)."""
-        if self.world == 1:
-            return
-        import torch.distributed as dist
-        padded = torch.zeros(self.per * self.world, dtype=t.dtype, device=t.device)
-        padded[:self.V] = t
-        out = list(padded.view(self.world, self.per).unbind(0))
-        dist.all_gather(out, padded[self.rank * self.per:(self.rank + 1) * self.per].clone(), group=self.group)
-        t.copy_(torch.stack(out).view(-1)[:self.V])
+        allgather_block(t, self.V, self.per, self.rank, self.world, self.group)
 
     def _allreduce_sum(self, t):
-        if self.world == 1:
-            return
-        import torch.distributed as dist
-        dist.all_reduce(t, group=self.group)
+        allreduce_sum(t, self.world, self.group)
 
     def _dispatch(self, method, objs_ptr, n, args, stream=None):
         st = self.ctx.dispatch_raw(self.v, vf.APP_GRAPH, method, objs_ptr, n, args, vf._stream(stream))

@@ -1,0 +1,221 @@
+#!/usr/bin/env python
+"""Measure every BASELINE.json config (beyond the config-2 headline in bench.py) on one B200.
+
+For each app, each dispatch variant: virtual calls/s over the timed steps
+(CUDA events on the launching stream, after warm-up), plus the algorithmic
+bytes (or FLOPs) per call and the fraction of the measured roof, and the CPU
+oracle timed on this host's cores on the same (or a stated sampled) input.
+Writes one JSON line per (app, variant) to <out>.jsonl and a table to <out>.md.
+
+  python tools/bench_apps.py --out profiles/apps_r1 [--apps gol,gen,graph,ray,traf] [--quick]
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+import oracle  # noqa: E402  (cpu_baseline leg only)
+import synth  # noqa: E402
+from paper_conf_asplos_zhangar21_b200 import apps, vf  # noqa: E402
+from paper_conf_asplos_zhangar21_b200.graph import Graph  # noqa: E402
+from paper_conf_asplos_zhangar21_b200.ray import Ray  # noqa: E402
+from paper_conf_asplos_zhangar21_b200.traf import Traf  # noqa: E402
+
+VARIANTS = ("cuda", "sharedoa", "coal", "typeptr")
+PEAKS = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))) if os.path.exists(
+    os.path.join(ROOT, "MEASURED_PEAKS.json")) else {}
+HBM = PEAKS.get("hbm_gbs", 6550.1)
+SMS = 148
+FP32_PEAK = SMS * 128 * 2 * PEAKS.get("sm_max_mhz", 1965.0) * 1e6 / 1e12  # TFLOP/s, derived
+ROWS = []
+
+
+def ev_time(fn, steps, warm=2):
+    for _ in range(warm):
+        fn()
+    torch.cuda.synchronize()
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record()
+    for _ in range(steps):
+        fn()
+    b.record()
+    torch.cuda.synchronize()
+    return a.elapsed_time(b) / steps
+
+
+def record(app, config, variant, calls_per_step, ms, unit_per_call, unit, bound, extra=None, cpu=None):
+    achieved = unit_per_call * calls_per_step / (ms / 1e3) / (1e9 if unit == "GB/s" else 1e12)
+    peak = HBM if unit == "GB/s" else FP32_PEAK
+    row = dict(app=app, config=config, variant=variant, calls_per_step=calls_per_step, ms_per_step=ms,
+               calls_per_s=calls_per_step / (ms / 1e3), roofline=dict(bound=bound, achieved=achieved, peak=peak,
+                                                                       unit=unit, frac=achieved / peak,
+                                                                       per_call=unit_per_call),
+               **(extra or {}))
+    if cpu:
+        row["cpu_baseline"] = cpu
+    ROWS.append(row)
+    print(json.dumps(row), flush=True)
+    return row
+
+
+def cpu_info(calls, sec, sample):
+    return dict(value=calls / sec, unit="calls/s", cores=oracle.max_threads(), kind="oracle", sample=sample)
+
+
+# ---------------------------------------------------------------- config 1: GOL
+def bench_gol(ctx, quick):
+    W = H = 256
+    gens = 100
+    g0 = synth.soup(W, H, seed=42)
+    _, _, _, sec = oracle.gol_run(W, H, g0, gens, threads=oracle.max_threads())
+    cpu = cpu_info(W * H * gens, sec, "full config (256x256, 100 generations)")
+    for v in VARIANTS:
+        g = apps.Gol(ctx, W, H, g0, v)
+        s = torch.cuda.Stream()
+        torch.cuda.synchronize()
+        graph = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(graph, stream=s):
+            for _ in range(gens):
+                g.gen(stream=s)
+        ms = ev_time(graph.replay, 5) / gens
+        ms_eager = ev_time(g.gen, 50)
+        # 8 B ptr + 1 B nbr + 1 B state out + 4 B counter r/w per next() call
+        record("gol", "256x256, 100 gens (CUDA graph of 100 generations)", v, W * H, ms, 14, "GB/s", "l2/latency",
+               dict(ms_per_gen_eager=ms_eager), cpu)
+        del g, graph
+    ctx.reset()
+
+
+# ---------------------------------------------------------------- config 5: GEN
+def bench_gen(ctx, quick):
+    W = H = 1024 if quick else 4096
+    gens = 20
+    s0 = synth.soup(W, H, seed=42)
+    _, _, _, sec = oracle.gen_run(W, H, s0, gens, threads=oracle.max_threads())
+    cpu = cpu_info(W * H * gens, sec, f"{W}x{H}, {gens} generations (same input)")
+    for v in VARIANTS:
+        Wv = W if v != "cuda" else min(W, 2048)  # device-heap new of 3 x 16.8M objects takes minutes
+        sv = s0 if Wv == W else synth.soup(Wv, Wv, seed=42)
+        g = apps.Gen(ctx, Wv, Wv, sv, v)
+        ms = ev_time(g.gen, gens)
+        record("gen", f"{Wv}x{Wv} B2/S345/C4", v, Wv * Wv, ms, 14, "GB/s", "hbm", None, cpu)
+        del g
+        ctx.reset()
+
+
+# ---------------------------------------------------------------- config 4: graph
+def bench_graph(ctx, quick):
+    scale = 20 if quick else 24
+    t0 = time.time()
+    offs, col = synth.rmat_graph(scale, seed=1)
+    print(f"# rmat-{scale}: V={len(offs) - 1} arcs={len(col)} gen {time.time() - t0:.1f}s", flush=True)
+    types = synth.vertex_types(offs)
+    src = int(np.argmax(np.diff(offs.astype(np.int64))))
+    V, arcs = len(offs) - 1, len(col)
+    thr = oracle.max_threads()
+    _, _, bcalls, bsec = oracle.graph_bfs(offs, col, types, src)
+    _, _, ccalls, csec = oracle.graph_cc(offs, col, types, threads=thr)
+    _, psec = oracle.graph_pr(offs, col, types, iters=5, threads=thr)
+    cpu = dict(bfs=cpu_info(bcalls, bsec, "full graph, 1 thread (sequential BFS)"),
+               cc=cpu_info(ccalls, csec, "full graph"),
+               pr=cpu_info(2 * V * 5, psec, "full graph, 5 iterations (2 virtual calls/vertex/iteration)"))
+    avg_deg = arcs / V
+    for v in VARIANTS:
+        g = Graph(ctx, offs, col, v)
+        ms = ev_time(lambda: g.bfs(src), 3, warm=1)
+        calls = g.calls
+        # per reached vertex: 8 B ptr + 8 B offs + per arc 4 B col + 4 B depth
+        record("graph-bfs", f"rmat-{scale} top-down BFS from max-degree vertex", v, calls, ms,
+               16 + 8 * avg_deg, "GB/s", "hbm", dict(V=V, arcs=arcs), cpu["bfs"])
+        ms = ev_time(lambda: g.cc(), 2, warm=1)
+        record("graph-cc", f"rmat-{scale} Jacobi CC to convergence", v, g.calls, ms, 20 + 8 * avg_deg, "GB/s",
+               "hbm", dict(iters=g.calls // V), cpu["cc"])
+        g.pr_init()
+        ms = ev_time(lambda: g.pr_iteration(), 10, warm=2)
+        # per vertex per iteration: contrib (8 ptr + 4 r + 8 c) and update (8 ptr + 8 offs + 4 out) + 8 B/arc
+        record("graph-pr", f"rmat-{scale} PageRank iteration", v, 2 * V, ms, (40 + 8 * avg_deg) / 2, "GB/s",
+               "hbm", None, cpu["pr"])
+        del g
+        ctx.reset()
+
+
+# ---------------------------------------------------------------- config 3: ray
+def bench_ray(ctx, quick):
+    W, H, S = (480, 270, 10000) if quick else (1920, 1080, 10000)
+    types, P = synth.ray_scene(S, seed=7)
+    cam = synth.ray_camera(W, H)
+    rows = 16 if not quick else 8
+    _, _, calls, sec = oracle.ray_render(W, H, types, P, cam, synth.RAY_ALBEDO, row0=H // 2 - rows // 2,
+                                         nrows=rows, threads=oracle.max_threads())
+    cpu = cpu_info(calls, sec, f"{rows} of {H} rows (centre band), full scene")
+    tcounts = np.bincount(types, minlength=4)
+    # formula FLOPs per hit() (fma = 2): plane 2, sphere 19, rect 12, triangle 51
+    flops = float((tcounts * np.array([2, 19, 12, 51])).sum() / S)
+    for v in VARIANTS:
+        r = Ray(ctx, types, P, v)
+        rgb = torch.empty((H, W, 3), dtype=torch.float32, device="cuda")
+        hid = torch.empty((H, W), dtype=torch.int32, device="cuda")
+        ms = ev_time(lambda: r.render(W, H, cam, rgb=rgb, hid=hid), 3, warm=1)
+        record("ray", f"{W}x{H}, {S} shapes, 1 primary ray/pixel", v, W * H * S, ms, flops, "TFLOP/s", "alu",
+               None, cpu)
+        del r
+        ctx.reset()
+
+
+# ---------------------------------------------------------------- config 5: TRAF
+def bench_traf(ctx, quick):
+    R, L = (400, 4096) if quick else (3277, 4096)
+    w = synth.traf_world(R, L, seed=11)
+    steps = 20
+    _, _, sec = oracle.traf_run(w, steps, threads=oracle.max_threads())
+    nveh = len(w["veh_ring"])
+    cpu = cpu_info((R * L + nveh) * steps, sec, f"full world, {steps} steps")
+    for v in VARIANTS:
+        t = Traf(ctx, w, v)
+        ms = ev_time(t.step, steps)
+        # cells: 8 ptr + 16 obj + 2 B writes; vehicles: 8 ptr + 24 obj r/w + ~6 B occupancy
+        per_call = (26 * R * L + 38 * nveh) / (R * L + nveh)
+        record("traf", f"{R} rings x {L} cells, {nveh} vehicles", v, t.calls_per_step, ms, per_call, "GB/s", "hbm",
+               dict(objects=R * L + nveh), cpu)
+        del t
+        ctx.reset()
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--apps", default="gol,ray,traf,gen,graph")
+    ap.add_argument("--out", default="gpurun_out/apps")
+    ap.add_argument("--quick", action="store_true")
+    a = ap.parse_args()
+    ctx = vf.Ctx(0, cuda_heap_bytes=16 << 30)
+    for name in a.apps.split(","):
+        globals()[f"bench_{name}"](ctx, a.quick)
+    os.makedirs(os.path.dirname(a.out) or ".", exist_ok=True)
+    with open(a.out + ".jsonl", "w") as f:
+        for r in ROWS:
+            f.write(json.dumps(r) + "\n")
+    with open(a.out + ".md", "w") as f:
+        f.write("| app | config | variant | calls/step | ms/step | Gcalls/s | vs cuda | achieved | frac | "
+                "oracle Gcalls/s (cores) |\n|---|---|---|---|---|---|---|---|---|---|\n")
+        for r in ROWS:
+            base = next((x for x in ROWS if x["app"] == r["app"] and x["variant"] == "cuda"), None)
+            rel = r["calls_per_s"] / base["calls_per_s"] if base else float("nan")
+            rf = r["roofline"]
+            cpu = r.get("cpu_baseline")
+            f.write(f"| {r['app']} | {r['config']} | {r['variant']} | {r['calls_per_step']} | {r['ms_per_step']:.3f} | "
+                    f"{r['calls_per_s'] / 1e9:.2f} | {rel:.2f} | {rf['achieved']:.1f} {rf['unit']} | {rf['frac']:.3f} | "
+                    f"{(cpu['value'] / 1e9) if cpu else float('nan'):.3f} ({cpu['cores'] if cpu else '-'}) |\n")
+    print("wrote", a.out)
+
+
+if __name__ == "__main__":
+    main()
