@@ -27,7 +27,7 @@ import numpy as np
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 SO = os.path.join(HERE, "liboracle.so")
-SOURCES = ["alloc.cpp", "micro.cpp", "gol.cpp", "gen.cpp", "graph.cpp", "ray.cpp", "traf.cpp"]
+SOURCES = ["alloc.cpp", "micro.cpp", "gol.cpp", "gen.cpp", "graph.cpp", "ray.cpp", "traf.cpp", "nbody.cpp"]
 NOT_FOUND = 0xFFFFFFFF
 
 
@@ -95,6 +95,9 @@ def lib():
         L.oracle_traf_run.restype = ctypes.c_int
         L.oracle_traf_run.argtypes = [U32, U32, U32, P, P, P, P, P, U32, U64, P, P, ctypes.c_int, P, P,
                                       ctypes.POINTER(ctypes.c_double)]
+        L.oracle_nbody_run.restype = ctypes.c_int
+        L.oracle_nbody_run.argtypes = [U32, P, P, P, U32, ctypes.c_float, P, ctypes.c_float, ctypes.c_int, P, P,
+                                       ctypes.POINTER(ctypes.c_double)]
         L.oracle_max_threads.restype = ctypes.c_int
         _lib = L
     return _lib
@@ -287,3 +290,21 @@ def traf_run(world: dict, steps: int, threads: int = 1):
     if rc:
         raise ValueError(f"oracle_traf_run rc={rc}")
     return pos, vel, sec.value
+
+
+def nbody_run(sys_: dict, steps: int, threads: int = 1):
+    """sys_ = synth.nbody_system(...); returns (pos float32[N,4], vel float32[N,3], seconds)."""
+    types = np.ascontiguousarray(sys_["types"], np.uint32)
+    pos = np.ascontiguousarray(sys_["pos"], np.float32)
+    vel = np.ascontiguousarray(sys_["vel"], np.float32)
+    eps2 = np.ascontiguousarray(sys_["eps2"], np.float32)
+    N = len(types)
+    po = np.zeros((N, 4), np.float32)
+    vo = np.zeros((N, 3), np.float32)
+    sec = ctypes.c_double()
+    rc = lib().oracle_nbody_run(N, types.ctypes.data, pos.ctypes.data, vel.ctypes.data, steps,
+                                ctypes.c_float(sys_["dt"]), eps2.ctypes.data, ctypes.c_float(sys_["damp"]), threads,
+                                po.ctypes.data, vo.ctypes.data, ctypes.byref(sec))
+    if rc:
+        raise ValueError(f"oracle_nbody_run rc={rc}")
+    return po, vo, sec.value

@@ -150,6 +150,15 @@ int oracle_traf_run(uint32_t R, uint32_t L, uint32_t nveh, const uint32_t* veh_r
                     const uint32_t* slow_thr, int threads, uint32_t* pos_out, uint32_t* v_out,
                     double* seconds);
 
+/* ---- Config 5 all-pairs N-body (reading G18; see nbody.cpp) -------------
+ * N bodies, types[i] in {0 Star, 1 Planet, 2 Dust}, pos4 = N x (x,y,z,m),
+ * vel3 = N x (vx,vy,vz); per step one virtual update() per body (softening
+ * eps2[type], Dust damped by `damp`), semi-implicit Euler with dt; outputs
+ * final positions (N x 4) and velocities (N x 3). */
+int oracle_nbody_run(uint32_t N, const uint32_t* types, const float* pos4, const float* vel3,
+                     uint32_t steps, float dt, const float* eps2, float damp, int threads,
+                     float* pos_out, float* vel_out, double* seconds);
+
 /* number of OpenMP threads actually available */
 int oracle_max_threads(void);
 

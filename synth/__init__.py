@@ -281,6 +281,29 @@ def traf_world(R: int, L: int, density: float = 0.25, light_p: float = 1.0 / 32,
                 seed=seed, vmax=TRAF_VMAX.copy(), slow_thr=slow_thr)
 
 
+# --------------------------------------------------------------------------
+# Config 5 N-body (reading G18)
+# --------------------------------------------------------------------------
+NBODY_EPS2 = np.array([0.05, 0.01, 0.002], np.float32)  # Star, Planet, Dust softening^2
+NBODY_MASS = ((5.0, 10.0), (0.5, 1.0), (0.01, 0.05))     # per-type mass ranges
+
+
+def nbody_system(N: int, seed: int = 10, dt: float = 1e-3, damp: float = 0.999):
+    """Bodies uniform in the unit-ish cube [-1,1]^3, velocities in [-0.1,0.1]^3,
+    type = uniform(3) (0 Star, 1 Planet, 2 Dust), mass uniform in the type's range."""
+    i = np.arange(N, dtype=np.uint64)
+    r = [_unit(seed, S_BODY, i * np.uint64(8) + np.uint64(k)) for k in range(8)]
+    types = uniform(draw(seed, S_BODY, i + np.uint64(1 << 40)), 3)
+    pos = np.zeros((N, 4), np.float32)
+    for k in range(3):
+        pos[:, k] = np.float32(2.0) * r[k] - np.float32(1.0)
+    lo = np.array([m[0] for m in NBODY_MASS], np.float32)[types]
+    hi = np.array([m[1] for m in NBODY_MASS], np.float32)[types]
+    pos[:, 3] = lo + r[3] * (hi - lo)
+    vel = np.stack([(np.float32(0.2) * r[4 + k] - np.float32(0.1)) for k in range(3)], 1).astype(np.float32)
+    return dict(types=types, pos=pos, vel=vel, eps2=NBODY_EPS2.copy(), dt=np.float32(dt), damp=np.float32(damp))
+
+
 # degree-bucket vertex types (SURVEY W6, reading G22): Leaf <=1, Low 2-15, Mid 16-255, Hub >=256
 DEG_BOUNDS = (1, 15, 255)
 
