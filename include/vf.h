@@ -44,6 +44,14 @@
 extern "C" {
 #endif
 
+/* float4 in the ABI: CUDA's float4 inside the library, a plain 16-B-aligned
+ * struct for C callers (same layout). */
+#if defined(__CUDACC__)
+typedef float4 float4_t;
+#else
+typedef struct { float x, y, z, w; } __attribute__((aligned(16))) float4_t;
+#endif
+
 typedef enum {
   VF_OK = 0,
   VF_ERR_INVALID = 1,         /* bad argument (null ctx, unknown app/method/type, ...) */
@@ -67,8 +75,30 @@ enum {
   VF_APP_GRAPH = 3, /* config 4: Vertex / Leaf / Low / Mid / Hub   (Table 2)  */
   VF_APP_RAY = 4,   /* config 3: Shape / Plane / Sphere / Rect / Triangle   */
   VF_APP_TRAF = 5,  /* config 5: Agent / PlainCell / LightCell / Car / Truck / Bus        */
-  VF_APP_COUNT = 6
+  VF_APP_NBODY = 6, /* config 5: Body / Star / Planet / Dust (all-pairs N-body, G18)      */
+  VF_APP_COUNT = 7
 };
+
+/* Methods of VF_APP_NBODY (reading G18; DynaSOAr's N-body, BASELINE north_star).
+ * Type ids 0 Star, 1 Planet, 2 Dust; constructor argument {u32 idx, f32 vx,
+ * vy, vz}. Positions+masses are float4 (x, y, z, m) arrays indexed by idx.
+ * update(): a = sum_{j != idx, ascending j} m_j d / (r^2+eps2[type])^{3/2}
+ * with r2 = fmaf(dx,dx,fmaf(dy,dy,fmaf(dz,dz,eps2))), 1/(r2*sqrt(r2)),
+ * a = fmaf(d, m_j*inv, a); Dust: v *= damp; v = fmaf(dt,a,v);
+ * pout[idx] = (fmaf(dt,v,x), ..., m). Reads pin[0..N), writes pout[idx]. */
+enum { VF_NBODY_UPDATE = 0, VF_NBODY_GET = 1 };
+typedef struct {
+  const float4_t* pin_dev;  /* N float4, positions at the start of the step (all bodies) */
+  float4_t* pout_dev;       /* N float4, this call writes pout[idx] of its bodies only   */
+  uint32_t N;
+  float dt;
+  float eps2[3];            /* per type softening^2                                      */
+  float damp;               /* Dust velocity factor per step                             */
+} vf_nbody_update_args;
+typedef struct {
+  float* vel_out_dev;       /* 3 floats per body at (idx - idx_base)                     */
+  uint32_t idx_base;
+} vf_nbody_get_args;
 
 /* Methods of VF_APP_TRAF (Table 2, reading G16). Type ids: 0
  * PlainCell, 1 LightCell (ctor arg {u32 cell, u32 phase}); 2 Car, 3 Truck,

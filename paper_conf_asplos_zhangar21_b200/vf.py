@@ -45,6 +45,19 @@ APP_TRAF = 5
 TRAF_CELL_UPDATE, TRAF_VEH_STEP, TRAF_GET, TRAF_PLACE = 0, 1, 2, 3
 
 
+APP_NBODY = 6
+NBODY_UPDATE, NBODY_GET = 0, 1
+
+
+class nbody_update_args(ctypes.Structure):
+    _fields_ = [("pin_dev", ctypes.c_void_p), ("pout_dev", ctypes.c_void_p), ("N", ctypes.c_uint32),
+                ("dt", ctypes.c_float), ("eps2", ctypes.c_float * 3), ("damp", ctypes.c_float)]
+
+
+class nbody_get_args(ctypes.Structure):
+    _fields_ = [("vel_out_dev", ctypes.c_void_p), ("idx_base", ctypes.c_uint32)]
+
+
 class traf_cell_args(ctypes.Structure):
     _fields_ = [("blocked_dev", ctypes.c_void_p), ("occ_next_dev", ctypes.c_void_p), ("t", ctypes.c_uint32)]
 

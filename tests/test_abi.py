@@ -86,3 +86,12 @@ def test_product_path_does_not_import_oracle():
             txt = open(os.path.join(ROOT, "oracle", f)).read()
             assert not re.search(r"^\s*(from|import)\s+paper_conf", txt, flags=re.M), f
             assert not re.search(r'#include\s+[<"].*vf(_internal)?\.h', txt), f
+
+
+def test_header_is_plain_c():
+    """include/vf.h compiles as C (and as C++) with no CUDA headers: the boundary
+    is plain pointers and sizes."""
+    for lang, std in (("c", "-std=c11"), ("c++", "-std=c++17")):
+        r = subprocess.run(["gcc", "-fsyntax-only", "-x", lang, std, "-Wall", "-Werror", HDR],
+                           capture_output=True, text=True)
+        assert r.returncode == 0, r.stderr
