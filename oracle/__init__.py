@@ -27,7 +27,7 @@ import numpy as np
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 SO = os.path.join(HERE, "liboracle.so")
-SOURCES = ["alloc.cpp", "micro.cpp", "gol.cpp", "gen.cpp", "graph.cpp", "ray.cpp", "traf.cpp", "nbody.cpp"]
+SOURCES = ["alloc.cpp", "micro.cpp", "gol.cpp", "gen.cpp", "graph.cpp", "ray.cpp", "traf.cpp", "nbody.cpp", "stut.cpp"]
 NOT_FOUND = 0xFFFFFFFF
 
 
@@ -98,6 +98,10 @@ def lib():
         L.oracle_nbody_run.restype = ctypes.c_int
         L.oracle_nbody_run.argtypes = [U32, P, P, P, U32, ctypes.c_float, P, ctypes.c_float, ctypes.c_int, P, P,
                                        ctypes.POINTER(ctypes.c_double)]
+        L.oracle_stut_run.restype = ctypes.c_int
+        F = ctypes.c_float
+        L.oracle_stut_run.argtypes = [U32, P, P, P, P, U32, P, P, P, P, P, P, U32, F, F, F, F, ctypes.c_int, P, P, P,
+                                      ctypes.POINTER(ctypes.c_double)]
         L.oracle_max_threads.restype = ctypes.c_int
         _lib = L
     return _lib
@@ -308,3 +312,26 @@ def nbody_run(sys_: dict, steps: int, threads: int = 1):
     if rc:
         raise ValueError(f"oracle_nbody_run rc={rc}")
     return po, vo, sec.value
+
+
+def stut_run(w: dict, steps: int, threads: int = 1):
+    """w = synth.stut_lattice(...) / synth.stut_custom(...); returns
+    (pos float32[n,2], vel float32[n,2], broken uint8[S], seconds). See oracle.h."""
+    n, S = len(w["types"]), len(w["a"])
+    c = lambda a, dt: np.ascontiguousarray(a, dtype=dt)
+    types, pos, vel, mass = c(w["types"], np.uint32), c(w["pos"], np.float32), c(w["vel"], np.float32), \
+        c(w["mass"], np.float32)
+    a, b, L0, k = c(w["a"], np.uint32), c(w["b"], np.uint32), c(w["L0"], np.float32), c(w["k"], np.float32)
+    io, inc = c(w["inc_offs"], np.uint32), c(w["inc"], np.uint32)
+    po = np.zeros((n, 2), np.float32)
+    vo = np.zeros((n, 2), np.float32)
+    bo = np.zeros(max(S, 1), np.uint8)
+    secs = ctypes.c_double(0)
+    rc = lib().oracle_stut_run(n, types.ctypes.data, pos.ctypes.data, vel.ctypes.data, mass.ctypes.data, S,
+                               a.ctypes.data, b.ctypes.data, L0.ctypes.data, k.ctypes.data, io.ctypes.data,
+                               inc.ctypes.data, steps, float(w["dt"]), float(w["damping"]), float(w["v_pull"]),
+                               float(w["break_ratio"]), threads, po.ctypes.data, vo.ctypes.data, bo.ctypes.data,
+                               ctypes.byref(secs))
+    if rc:
+        raise ValueError(f"oracle_stut_run rc={rc}")
+    return po, vo, bo[:S], secs.value

@@ -159,6 +159,18 @@ int oracle_nbody_run(uint32_t N, const uint32_t* types, const float* pos4, const
                      uint32_t steps, float dt, const float* eps2, float damp, int threads,
                      float* pos_out, float* vel_out, double* seconds);
 
+/* ---- Config 5 STUT spring-node structure (reading G17; see stut.cpp) ----
+ * n nodes (types 0 Node, 1 AnchorNode, 2 AnchorPullNode; pos2 / vel2 = n x 2,
+ * mass), S springs (sa, sb, rest L0, stiffness k), incidence CSR (inc_offs[n+1],
+ * inc = (spring << 1) | is_b_end, ascending spring id per node). Per step: a
+ * virtual force() per spring, then a virtual move() per node. Outputs final
+ * positions / velocities (n x 2) and the broken flag per spring. */
+int oracle_stut_run(uint32_t n, const uint32_t* types, const float* pos2, const float* vel2,
+                    const float* mass, uint32_t S, const uint32_t* sa, const uint32_t* sb,
+                    const float* L0, const float* k, const uint32_t* inc_offs, const uint32_t* inc,
+                    uint32_t steps, float dt, float c, float v_pull, float brk, int threads,
+                    float* pos_out, float* vel_out, uint8_t* broken_out, double* seconds);
+
 /* number of OpenMP threads actually available */
 int oracle_max_threads(void);
 

@@ -39,9 +39,10 @@ def allgather_block(t, V: int, per: int, rank: int, world: int, group=None):
     if world == 1:
         return
     import torch.distributed as dist
-    padded = torch.zeros(per * world, dtype=t.dtype, device=t.device)
+    rest = tuple(t.shape[1:])  # per-vertex rows (e.g. float4 positions)
+    padded = torch.zeros((per * world,) + rest, dtype=t.dtype, device=t.device)
     padded[:V] = t
-    out = [torch.empty(per, dtype=t.dtype, device=t.device) for _ in range(world)]
+    out = [torch.empty((per,) + rest, dtype=t.dtype, device=t.device) for _ in range(world)]
     dist.all_gather(out, padded[rank * per:(rank + 1) * per].clone(), group=group)
     t.copy_(torch.cat(out)[:V])
 

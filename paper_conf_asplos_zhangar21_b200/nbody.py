@@ -22,7 +22,7 @@ from .graph import allgather_block, block_range
 
 class Nbody:
     def __init__(self, ctx: vf.Ctx, sys_: dict, variant: str = "typeptr", rank: int = 0, world: int = 1,
-                 group=None):
+                 group=None, exchange: bool = True):
         self.ctx, self.variant = ctx, variant
         self.v = vf.VARIANTS[variant]
         dev = torch.device(f"cuda:{ctx.device}")
@@ -30,6 +30,7 @@ class Nbody:
         N = len(sys_["types"])
         self.N = N
         self.rank, self.world, self.group = rank, world, group
+        self.exchange = exchange  # False: the caller stitches the owned slices (emulated ranks)
         self.lo, self.hi, self.per = block_range(N, rank, world)
         own = np.arange(self.lo, self.hi)
         ctor = np.zeros((len(own), 4), np.uint32)
@@ -62,7 +63,7 @@ class Nbody:
                                    self.hi - self.lo, self._args(), s)
         if st:
             self.ctx._check(st, "nbody update")
-        if self.world > 1:
+        if self.world > 1 and self.exchange:
             allgather_block(self.p[1], self.N, self.per, self.rank, self.world, self.group)
         self.p[0], self.p[1] = self.p[1], self.p[0]
 

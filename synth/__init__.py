@@ -311,3 +311,79 @@ DEG_BOUNDS = (1, 15, 255)
 def vertex_types(offs) -> np.ndarray:
     deg = np.diff(np.asarray(offs, dtype=np.int64))
     return np.digitize(deg, [DEG_BOUNDS[0] + 1, DEG_BOUNDS[1] + 1, DEG_BOUNDS[2] + 1]).astype(np.uint32)
+
+
+# --------------------------------------------------------------------------
+# Config 5 STUT spring-node structure (reading G17)
+# --------------------------------------------------------------------------
+STUT_NODE, STUT_ANCHOR, STUT_PULL, STUT_SPRING = 0, 1, 2, 3  # type ids
+
+
+def stut_lattice(W: int, H: int, seed: int = 12, jitter: float = 0.1, k0: float = 20.0, dt: float = 0.01,
+                 damping: float = 0.05, v_pull: float = 1.0, break_ratio: float = 1.5):
+    """W x H node lattice, node n = y*W + x at (x, y) (+ seeded jitter for free
+    nodes); column 0 = AnchorNode, column W-1 = AnchorPullNode, else Node;
+    mass 1 + 0.5u. Springs in the order (y, x, {right, down, diagonal}) with
+    rest length 1 (axis) or float32(sqrt 2) (diagonal), stiffness k0(0.5+u).
+    Incidence (structure only): for every node the springs touching it in
+    ascending spring id, code = (spring << 1) | (node is the spring's b end)."""
+    n = W * H
+    i = np.arange(n, dtype=np.uint64)
+    x = (np.arange(n) % W).astype(np.float32)
+    y = (np.arange(n) // W).astype(np.float32)
+    types = np.full(n, STUT_NODE, np.uint32)
+    types[np.arange(n) % W == 0] = STUT_ANCHOR
+    types[np.arange(n) % W == W - 1] = STUT_PULL
+    free = types == STUT_NODE
+    jx = np.float32(jitter) * (np.float32(2.0) * _unit(seed, S_STUT, 4 * i) - np.float32(1.0))
+    jy = np.float32(jitter) * (np.float32(2.0) * _unit(seed, S_STUT, 4 * i + np.uint64(1)) - np.float32(1.0))
+    pos = np.stack([np.where(free, x + jx, x), np.where(free, y + jy, y)], 1).astype(np.float32)
+    mass = (np.float32(1.0) + np.float32(0.5) * _unit(seed, S_STUT, 4 * i + np.uint64(2))).astype(np.float32)
+    a, b, L0 = [], [], []
+    nodes = np.arange(n, dtype=np.int64).reshape(H, W)
+    diag = np.float32(np.sqrt(2.0))
+    # enumerate (y, x, kind) in order via a [H, W, 3] table, -1 = absent
+    tab_b = np.full((H, W, 3), -1, np.int64)
+    tab_b[:, :-1, 0] = nodes[:, 1:]
+    tab_b[:-1, :, 1] = nodes[1:, :]
+    tab_b[:-1, :-1, 2] = nodes[1:, 1:]
+    tab_a = np.broadcast_to(nodes[:, :, None], (H, W, 3))
+    kind = np.broadcast_to(np.arange(3)[None, None, :], (H, W, 3))
+    sel = tab_b.reshape(-1) >= 0
+    a = tab_a.reshape(-1)[sel].astype(np.uint32)
+    b = tab_b.reshape(-1)[sel].astype(np.uint32)
+    L0 = np.where(kind.reshape(-1)[sel] == 2, diag, np.float32(1.0)).astype(np.float32)
+    S = len(a)
+    si = np.arange(S, dtype=np.uint64)
+    k = (np.float32(k0) * (np.float32(0.5) + _unit(seed, S_STUT, (si << np.uint64(2)) + np.uint64(3)
+                                                   + np.uint64(1 << 40)))).astype(np.float32)
+    inc_offs, inc = stut_incidence(n, a, b)
+    return dict(W=W, H=H, types=types, pos=pos, vel=np.zeros((n, 2), np.float32), mass=mass, a=a, b=b, L0=L0,
+                k=k, inc_offs=inc_offs, inc=inc, dt=np.float32(dt), damping=np.float32(damping),
+                v_pull=np.float32(v_pull), break_ratio=np.float32(break_ratio))
+
+
+def stut_incidence(n: int, a: np.ndarray, b: np.ndarray):
+    """CSR of the springs touching each node, ascending spring id; code =
+    (s << 1) | is_b. Pure structure (no method arithmetic)."""
+    S = len(a)
+    s = np.arange(S, dtype=np.uint64)
+    node = np.concatenate([np.asarray(a, np.int64), np.asarray(b, np.int64)])
+    code = np.concatenate([s << np.uint64(1), (s << np.uint64(1)) | np.uint64(1)]).astype(np.uint32)
+    order = np.lexsort((code, node))
+    offs = np.zeros(n + 1, np.uint32)
+    np.add.at(offs, node + 1, 1)
+    return np.cumsum(offs).astype(np.uint32), code[order]
+
+
+def stut_custom(types, pos, mass, a, b, L0, k, vel=None, dt=0.01, damping=0.0, v_pull=1.0, break_ratio=1.5):
+    """A hand-built structure (tests): same dict as stut_lattice."""
+    n = len(types)
+    a = np.asarray(a, np.uint32)
+    b = np.asarray(b, np.uint32)
+    inc_offs, inc = stut_incidence(n, a, b)
+    return dict(W=n, H=1, types=np.asarray(types, np.uint32), pos=np.asarray(pos, np.float32).reshape(n, 2),
+                vel=(np.zeros((n, 2), np.float32) if vel is None else np.asarray(vel, np.float32).reshape(n, 2)),
+                mass=np.asarray(mass, np.float32), a=a, b=b, L0=np.asarray(L0, np.float32),
+                k=np.asarray(k, np.float32), inc_offs=inc_offs, inc=inc, dt=np.float32(dt),
+                damping=np.float32(damping), v_pull=np.float32(v_pull), break_ratio=np.float32(break_ratio))

@@ -62,7 +62,7 @@ def test_nbody_block_shards_reassemble(ctx):
     N, steps, world = 777, 3, 3
     s = synth.nbody_system(N, seed=9)
     p_ref, v_ref, _ = oracle.nbody_run(s, steps)
-    ranks = [Nbody(ctx, s, "coal", r, world) for r in range(world)]
+    ranks = [Nbody(ctx, s, "coal", r, world, exchange=False) for r in range(world)]
     for _ in range(steps):
         for nb in ranks:
             nb.step()
