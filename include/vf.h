@@ -48,8 +48,10 @@ extern "C" {
  * struct for C callers (same layout). */
 #if defined(__CUDACC__)
 typedef float4 float4_t;
+typedef float2 float2_t;
 #else
 typedef struct { float x, y, z, w; } __attribute__((aligned(16))) float4_t;
+typedef struct { float x, y; } __attribute__((aligned(8))) float2_t;
 #endif
 
 typedef enum {
@@ -76,8 +78,40 @@ enum {
   VF_APP_RAY = 4,   /* config 3: Shape / Plane / Sphere / Rect / Triangle   */
   VF_APP_TRAF = 5,  /* config 5: Agent / PlainCell / LightCell / Car / Truck / Bus        */
   VF_APP_NBODY = 6, /* config 5: Body / Star / Planet / Dust (all-pairs N-body, G18)      */
-  VF_APP_COUNT = 7
+  VF_APP_STUT = 7,  /* config 5: Element / Node / AnchorNode / AnchorPullNode / Spring   */
+  VF_APP_COUNT = 8
 };
+
+/* Methods of VF_APP_STUT (Table 2 "structure" P:1524-1528, reading G17). Type
+ * ids 0 Node, 1 AnchorNode, 2 AnchorPullNode (ctor {u32 id, f32 vx, vy, m}),
+ * 3 Spring (ctor {u32 id, a, b, f32 L0, k, u32 pad}). One step = FORCE on
+ * every spring, then MOVE on every node:
+ *   force(): broken -> 0; d = pos[b]-pos[a], len = sqrt(fmaf(dx,dx,dy*dy));
+ *            len > break_ratio*L0 -> broken = 1 (permanent), 0; else
+ *            fs = (k*(len-L0))/len, F[id] = (fs*dx, fs*dy) (acts on a, -F on b)
+ *   move():  Node: sum F of incident springs (inc_offs/inc CSR, code =
+ *            spring<<1 | is_b, ascending), F = fmaf(-c, v, F),
+ *            v = fmaf(dt, F/m, v), pos = fmaf(dt, v, pos); AnchorNode: none;
+ *            AnchorPullNode: pos.x = fmaf(dt, v_pull, pos.x).
+ * Methods a class does not define are no-ops on it. */
+enum { VF_STUT_FORCE = 0, VF_STUT_MOVE = 1, VF_STUT_GET = 2 };
+typedef struct {
+  const float2_t* pos_dev;  /* node positions (n)                 */
+  float2_t* F_dev;          /* per-spring force of this step (S)  */
+  float break_ratio;
+} vf_stut_force_args;
+typedef struct {
+  float2_t* pos_dev;
+  const float2_t* F_dev;
+  const uint32_t* inc_offs_dev;  /* n+1 */
+  const uint32_t* inc_dev;       /* 2S  */
+  float dt, c, v_pull;
+} vf_stut_move_args;
+typedef struct {
+  float* vel_out_dev;       /* nodes: 2 floats at (id - id_base), may be NULL      */
+  uint8_t* broken_out_dev;  /* springs: flag at (id - spring_base), may be NULL    */
+  uint32_t id_base, spring_base;
+} vf_stut_get_args;
 
 /* Methods of VF_APP_NBODY (reading G18; DynaSOAr's N-body, BASELINE north_star).
  * Type ids 0 Star, 1 Planet, 2 Dust; constructor argument {u32 idx, f32 vx,

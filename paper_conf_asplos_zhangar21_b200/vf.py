@@ -58,6 +58,25 @@ class nbody_get_args(ctypes.Structure):
     _fields_ = [("vel_out_dev", ctypes.c_void_p), ("idx_base", ctypes.c_uint32)]
 
 
+APP_STUT = 7
+STUT_FORCE, STUT_MOVE, STUT_GET = 0, 1, 2
+
+
+class stut_force_args(ctypes.Structure):
+    _fields_ = [("pos_dev", ctypes.c_void_p), ("F_dev", ctypes.c_void_p), ("break_ratio", ctypes.c_float)]
+
+
+class stut_move_args(ctypes.Structure):
+    _fields_ = [("pos_dev", ctypes.c_void_p), ("F_dev", ctypes.c_void_p), ("inc_offs_dev", ctypes.c_void_p),
+                ("inc_dev", ctypes.c_void_p), ("dt", ctypes.c_float), ("c", ctypes.c_float),
+                ("v_pull", ctypes.c_float)]
+
+
+class stut_get_args(ctypes.Structure):
+    _fields_ = [("vel_out_dev", ctypes.c_void_p), ("broken_out_dev", ctypes.c_void_p), ("id_base", ctypes.c_uint32),
+                ("spring_base", ctypes.c_uint32)]
+
+
 class traf_cell_args(ctypes.Structure):
     _fields_ = [("blocked_dev", ctypes.c_void_p), ("occ_next_dev", ctypes.c_void_p), ("t", ctypes.c_uint32)]
 
