@@ -194,27 +194,42 @@ typedef struct { uint16_t* counter_out_dev; uint8_t* type_out_dev; } vf_gen_get_
 /* Methods of VF_APP_GRAPH (readings G20-G23). Type ids by degree: 0 Leaf
  * (<= 1), 1 Low (2..15), 2 Mid (16..255), 3 Hub (>= 256). Constructor
  * argument per object: { u32 vid, u32 deg }. CSR: offs[V+1] (u64), col (u32),
- * symmetric. vobj_dev[v] = the object pointer of vertex v. */
+ * symmetric. vobj_dev[v] = the object pointer of vertex v.
+ *
+ * Work entries (load balance): a dispatch list holds one entry
+ * per (vertex, edge chunk): a vertex of degree deg > C appears
+ * nch = ceil(deg / C) times, consecutively, with chunk_dev[i] = 0 .. nch-1
+ * (chunk_dev is read only for such vertices); every other vertex appears once.
+ * Entry i of vertex v covers edges [offs[v] + c*C, min(offs[v] + (c+1)*C,
+ * offs[v+1])). Each entry is one virtual call on v's object. */
 enum {
   VF_GRAPH_BFS_EXPAND = 0, /* top-down: claim depth[u] = level+1 for unvisited neighbours
-                              (atomicCAS) and append vobj[u] to next_queue            */
+                              (atomicCAS) and append u's entries to next_queue /
+                              next_chunk; *next_count counts appended entries           */
   VF_GRAPH_BFS_PROBE = 1,  /* bottom-up: an unvisited vertex with a neighbour at `level`
-                              takes depth level+1; next_count counts them               */
-  VF_GRAPH_CC_UPDATE = 2,  /* label_out[v] = min(label_in over v and N(v)); changed = 1
-                              if it differs from label_in[v] (Jacobi)                   */
-  VF_GRAPH_PR_CONTRIB = 3, /* contrib[v] = deg ? rank_in[v]/deg : 0 (fp64); deg-0
-                              vertices add rank_in[v] to *dangling                       */
+                              takes depth level+1 (atomicCAS); *next_count = 1 if any   */
+  VF_GRAPH_CC_UPDATE = 2,  /* label_out[v] = min(label_in over v and N(v)) (Jacobi; a
+                              multi-chunk vertex combines with atomicMin: label_out must
+                              hold a label >= label_in[v], e.g. the previous-but-one
+                              iterate); *changed = 1 if it is below label_in[v]          */
+  VF_GRAPH_PR_CONTRIB = 3, /* chunk 0 only: contrib[v] = deg ? rank_in[v]/deg : 0 (fp64);
+                              deg-0 vertices add rank_in[v] to *dangling                 */
   VF_GRAPH_PR_UPDATE = 4   /* rank_out[v] = (float)(base + d*(sum_{N(v)} contrib +
-                              *dangling / Vd)), base = (1-d)/V                          */
+                              *dangling / Vd)); a multi-chunk vertex writes its chunk sum
+                              to partial[i]; the last chunk to finish (counter[v]) sums
+                              the partials in chunk order and resets counter[v] to 0    */
 };
 typedef struct {
   const uint64_t* offs_dev;
   const uint32_t* col_dev;
   int32_t* depth_dev;
   const uint64_t* vobj_dev;
-  uint64_t* next_queue_dev;
+  const uint32_t* chunk_dev;   /* chunk index of each entry of this dispatch       */
+  uint64_t* next_queue_dev;    /* top-down: next frontier entries (objects)        */
+  uint32_t* next_chunk_dev;    /* top-down: their chunk indices                    */
   uint32_t* next_count_dev;
   int32_t level;
+  uint32_t C;                  /* edges per chunk (>= 1)                           */
 } vf_graph_bfs_args;
 typedef struct {
   const uint64_t* offs_dev;
@@ -222,6 +237,8 @@ typedef struct {
   const uint32_t* label_in_dev;
   uint32_t* label_out_dev;
   uint32_t* changed_dev;
+  const uint32_t* chunk_dev;
+  uint32_t C;
 } vf_graph_cc_args;
 typedef struct {
   const uint64_t* offs_dev;
@@ -231,6 +248,10 @@ typedef struct {
   double* contrib_dev;
   double* dangling_dev;
   double base, d, Vd;
+  const uint32_t* chunk_dev;
+  double* partial_dev;         /* one slot per entry of this dispatch              */
+  uint32_t* counter_dev;       /* per vertex, zero between iterations              */
+  uint32_t C;
 } vf_graph_pr_args;
 
 #define VF_MAX_RANGES 4096u     /* COAL range-table capacity (staged in shared memory)   */
@@ -385,9 +406,11 @@ vf_status vf_ray_render(vf_ctx* ctx, vf_variant v, const uint64_t* shapes_dev, u
                         float* rgb_dev, int32_t* hit_dev, void* stream);
 
 /* Graph helpers: BFS start state (depth = -1 except depth[src] = 0, queue =
- * [vobj[src]], *count = 1), iota (x[i] = i), fill (x[i] = value). */
+ * src's nch work entries (vobj[src], chunks 0..nch-1), *count = nch), iota
+ * (x[i] = i), fill (x[i] = value). */
 vf_status vf_graph_bfs_init(uint64_t V, int32_t* depth_dev, uint32_t src, const uint64_t* vobj_dev,
-                            uint64_t* queue_dev, uint32_t* count_dev, void* stream);
+                            const uint64_t* offs_dev, uint32_t C, uint64_t* queue_dev,
+                            uint32_t* queue_chunk_dev, uint32_t* count_dev, void* stream);
 vf_status vf_iota_u32(uint64_t n, uint32_t* x_dev, void* stream);
 vf_status vf_fill_f32(uint64_t n, float* x_dev, float value, void* stream);
 

@@ -5,6 +5,10 @@
 // implement the same semantics (the oracle's plain loops); each picks the
 // loop shape that suits its degree: Leaf has no loop, Low a plain loop, Mid
 // and Hub unrolled loops with independent accumulators (more loads in flight).
+// High-degree vertices are split into work entries of <= C edges (vf.h), so no
+// lane walks a hub's whole row. (Measured on B200: sharing one member's row
+// across the group's lanes in turn — coalesced but serial per vertex — was
+// 1.2-1.5x SLOWER than these per-lane loops at RMAT-24.)
 //
 // Object layout (16 B): { vTable* (8 B), u32 vid, u32 deg }.
 #include "dispatch.cuh"
@@ -21,11 +25,12 @@ struct Vertex {
       : vid(arg ? static_cast<const CtorArg*>(arg)->vid : 0),
         deg(arg ? static_cast<const CtorArg*>(arg)->deg : 0) {}
   __device__ virtual ~Vertex() {}
-  __device__ virtual void bfs_expand(vf_graph_bfs_args a) = 0;
-  __device__ virtual void bfs_probe(vf_graph_bfs_args a) = 0;
-  __device__ virtual void cc_update(vf_graph_cc_args a) = 0;
-  __device__ virtual void pr_contrib(vf_graph_pr_args a) = 0;
-  __device__ virtual void pr_update(vf_graph_pr_args a) = 0;
+  // i = index of this call's work entry in the dispatched array (its chunk)
+  __device__ virtual void bfs_expand(vf_graph_bfs_args a, uint64_t i) = 0;
+  __device__ virtual void bfs_probe(vf_graph_bfs_args a, uint64_t i) = 0;
+  __device__ virtual void cc_update(vf_graph_cc_args a, uint64_t i) = 0;
+  __device__ virtual void pr_contrib(vf_graph_pr_args a, uint64_t i) = 0;
+  __device__ virtual void pr_update(vf_graph_pr_args a, uint64_t i) = 0;
   uint32_t vid;
   uint32_t deg;
 };
@@ -46,78 +51,141 @@ __device__ __forceinline__ void for_neighbors(const uint32_t* __restrict__ col, 
   for (; k < e; ++k) f(__ldg(col + k));
 }
 
+__device__ __forceinline__ uint32_t nchunks(uint32_t deg, uint32_t C) { return deg <= C ? 1u : (deg + C - 1) / C; }
+
+// The edge range of work entry i of vertex (vid, deg): chunk c of <= C edges.
+// Single-chunk vertices (deg <= C, nearly all) never read the chunk array.
+struct Work {
+  uint64_t b, e;
+  uint32_t c, nch;
+};
+__device__ __forceinline__ Work work_of(const uint64_t* offs, const uint32_t* chunk, uint64_t i, uint32_t vid,
+                                        uint32_t deg, uint32_t C) {
+  Work w;
+  w.nch = nchunks(deg, C);
+  w.c = w.nch > 1 ? __ldg(chunk + i) : 0u;
+  const uint64_t b0 = __ldg(offs + vid);
+  w.b = b0 + (uint64_t)w.c * C;
+  const uint64_t e0 = b0 + deg;
+  w.e = w.b + C < e0 ? w.b + C : e0;
+  return w;
+}
+
+// Append vertex u's work entries to the next BFS frontier. Single-chunk
+// vertices reserve their slots with one warp-aggregated atomic per group of
+// lanes that claim at the same time, multi-chunk ones alone.
+__device__ __forceinline__ void enqueue(const vf_graph_bfs_args& a, uint32_t u) {
+  const uint32_t d = (uint32_t)(__ldg(a.offs_dev + u + 1) - __ldg(a.offs_dev + u));
+  const uint32_t n = nchunks(d, a.C);
+  const uint64_t obj = __ldg(a.vobj_dev + u);
+  if (n == 1) {
+    const uint32_t m = __activemask();
+    const uint32_t lane = threadIdx.x & 31u;
+    const uint32_t leader = __ffs(m) - 1;
+    uint32_t base = 0;
+    if (lane == leader) base = atomicAdd(a.next_count_dev, (uint32_t)__popc(m));
+    base = __shfl_sync(m, base, leader) + __popc(m & ((1u << lane) - 1u));
+    a.next_queue_dev[base] = obj;
+    a.next_chunk_dev[base] = 0;
+  } else {
+    const uint32_t base = atomicAdd(a.next_count_dev, n);
+    for (uint32_t j = 0; j < n; ++j) {
+      a.next_queue_dev[base + j] = obj;
+      a.next_chunk_dev[base + j] = j;
+    }
+  }
+}
+
 template <int KIND>
 struct VertexK final : Vertex {
   static constexpr int U = KIND == 0 ? 1 : KIND == 1 ? 1 : KIND == 2 ? 4 : 8;
   __device__ explicit VertexK(const void* arg) : Vertex(arg) {}
 
-  __device__ void bfs_expand(vf_graph_bfs_args a) override {
-    const uint64_t b = a.offs_dev[vid];
-    for_neighbors<U>(a.col_dev, b, b + deg, [&](uint32_t u) {
-      if (a.depth_dev[u] == -1 && atomicCAS(a.depth_dev + u, -1, a.level + 1) == -1)
-        a.next_queue_dev[atomicAdd(a.next_count_dev, 1u)] = a.vobj_dev[u];
+  __device__ void bfs_expand(vf_graph_bfs_args a, uint64_t i) {
+    const Work w = work_of(a.offs_dev, a.chunk_dev, i, vid, deg, a.C);
+    for_neighbors<U>(a.col_dev, w.b, w.e, [&](uint32_t u) {
+      if (a.depth_dev[u] == -1 && atomicCAS(a.depth_dev + u, -1, a.level + 1) == -1) enqueue(a, u);
     });
   }
   // bottom-up step: an unvisited vertex joins level+1 if a neighbour is at `level`
-  __device__ void bfs_probe(vf_graph_bfs_args a) override {
-    if (a.depth_dev[vid] != -1) return;
-    const uint64_t b = a.offs_dev[vid];
-    for (uint64_t k = b; k < b + deg; ++k) {
+  __device__ void bfs_probe(vf_graph_bfs_args a, uint64_t i) {
+    if (*(volatile int32_t*)(a.depth_dev + vid) != -1) return;
+    const Work w = work_of(a.offs_dev, a.chunk_dev, i, vid, deg, a.C);
+    for (uint64_t k = w.b; k < w.e; ++k) {
       if (a.depth_dev[__ldg(a.col_dev + k)] == a.level) {
-        a.depth_dev[vid] = a.level + 1;
-        atomicAdd(a.next_count_dev, 1u);
+        if (atomicCAS(a.depth_dev + vid, -1, a.level + 1) == -1) *(volatile uint32_t*)a.next_count_dev = 1u;
         return;
       }
     }
   }
-  __device__ void cc_update(vf_graph_cc_args a) override {
-    const uint32_t own = a.label_in_dev[vid];
+  __device__ void cc_update(vf_graph_cc_args a, uint64_t i) {
+    const Work w = work_of(a.offs_dev, a.chunk_dev, i, vid, deg, a.C);
+    const uint32_t own = __ldg(a.label_in_dev + vid);
     uint32_t m = own;
-    const uint64_t b = a.offs_dev[vid];
     if constexpr (U == 1) {
-      for_neighbors<1>(a.col_dev, b, b + deg, [&](uint32_t u) { m = min(m, __ldg(a.label_in_dev + u)); });
+      for_neighbors<1>(a.col_dev, w.b, w.e, [&](uint32_t u) { m = min(m, __ldg(a.label_in_dev + u)); });
     } else {
       uint32_t acc[U];
 #pragma unroll
       for (int j = 0; j < U; ++j) acc[j] = own;
-      uint64_t k = b;
-      const uint64_t e = b + deg;
-      for (; k + U <= e; k += U) {
+      uint64_t k = w.b;
+      for (; k + U <= w.e; k += U) {
 #pragma unroll
         for (int j = 0; j < U; ++j) acc[j] = min(acc[j], __ldg(a.label_in_dev + __ldg(a.col_dev + k + j)));
       }
-      for (; k < e; ++k) acc[0] = min(acc[0], __ldg(a.label_in_dev + __ldg(a.col_dev + k)));
+      for (; k < w.e; ++k) acc[0] = min(acc[0], __ldg(a.label_in_dev + __ldg(a.col_dev + k)));
 #pragma unroll
       for (int j = 0; j < U; ++j) m = min(m, acc[j]);
     }
-    a.label_out_dev[vid] = m;
+    if (w.nch == 1) a.label_out_dev[vid] = m;
+    else atomicMin(a.label_out_dev + vid, m);
     if (m != own) a.changed_dev[0] = 1u;
   }
-  __device__ void pr_contrib(vf_graph_pr_args a) override {
+  __device__ void pr_contrib(vf_graph_pr_args a, uint64_t i) {
+    if (nchunks(deg, a.C) > 1 && __ldg(a.chunk_dev + i) != 0) return;  // once per vertex
     const float r = a.rank_in_dev[vid];
     a.contrib_dev[vid] = deg ? (double)r / (double)deg : 0.0;
-    if (!deg) atomicAdd(a.dangling_dev, (double)r);
+    if (!deg) {
+      // dangling mass: one fp64 atomic per group of lanes that get here together
+      // (RMAT graphs have millions of isolated vertices: per-lane atomics on one
+      // address serialise in L2); the group sum is taken in lane order
+      const uint32_t m = __activemask();
+      const double x = (double)r;
+      double total = 0.0;
+      for (uint32_t mm = m; mm; mm &= mm - 1) total += __shfl_sync(m, x, __ffs(mm) - 1);
+      if ((threadIdx.x & 31u) == (uint32_t)(__ffs(m) - 1)) atomicAdd(a.dangling_dev, total);
+    }
   }
-  __device__ void pr_update(vf_graph_pr_args a) override {
-    const uint64_t b = a.offs_dev[vid];
+  __device__ void pr_update(vf_graph_pr_args a, uint64_t i) {
+    const Work w = work_of(a.offs_dev, a.chunk_dev, i, vid, deg, a.C);
     double s;
     if constexpr (U == 1) {
       s = 0.0;
-      for_neighbors<1>(a.col_dev, b, b + deg, [&](uint32_t u) { s += __ldg(a.contrib_dev + u); });
+      for_neighbors<1>(a.col_dev, w.b, w.e, [&](uint32_t u) { s += __ldg(a.contrib_dev + u); });
     } else {
       double acc[U];
 #pragma unroll
       for (int j = 0; j < U; ++j) acc[j] = 0.0;
-      uint64_t k = b;
-      const uint64_t e = b + deg;
-      for (; k + U <= e; k += U) {
+      uint64_t k = w.b;
+      for (; k + U <= w.e; k += U) {
 #pragma unroll
         for (int j = 0; j < U; ++j) acc[j] += __ldg(a.contrib_dev + __ldg(a.col_dev + k + j));
       }
-      for (; k < e; ++k) acc[0] += __ldg(a.contrib_dev + __ldg(a.col_dev + k));
+      for (; k < w.e; ++k) acc[0] += __ldg(a.contrib_dev + __ldg(a.col_dev + k));
       s = 0.0;
 #pragma unroll
       for (int j = 0; j < U; ++j) s += acc[j];
+    }
+    if (w.nch > 1) {
+      // last-finisher combine, in chunk order (deterministic)
+      a.partial_dev[i] = s;
+      __threadfence();
+      if (atomicAdd(a.counter_dev + vid, 1u) != w.nch - 1) return;
+      __threadfence();
+      const uint64_t first = i - w.c;
+      s = 0.0;
+      for (uint32_t j = 0; j < w.nch; ++j) s += __ldcg(a.partial_dev + first + j);
+      a.counter_dev[vid] = 0;
     }
     const double D = *a.dangling_dev;
     // (1-d)/V + d*(s + D/V), the oracle's operation order, IEEE fp64 (no contraction)
@@ -136,20 +204,20 @@ struct App {
   using Type = VertexK<K>;
 
   template <int M>
-  __device__ __forceinline__ static void vcall(Base* o, uint64_t, const ArgBlob& b) {
-    if constexpr (M == VF_GRAPH_BFS_EXPAND) o->bfs_expand(blob_as<vf_graph_bfs_args>(b));
-    else if constexpr (M == VF_GRAPH_BFS_PROBE) o->bfs_probe(blob_as<vf_graph_bfs_args>(b));
-    else if constexpr (M == VF_GRAPH_CC_UPDATE) o->cc_update(blob_as<vf_graph_cc_args>(b));
-    else if constexpr (M == VF_GRAPH_PR_CONTRIB) o->pr_contrib(blob_as<vf_graph_pr_args>(b));
-    else o->pr_update(blob_as<vf_graph_pr_args>(b));
+  __device__ __forceinline__ static void vcall(Base* o, uint64_t i, const ArgBlob& b) {
+    if constexpr (M == VF_GRAPH_BFS_EXPAND) o->bfs_expand(blob_as<vf_graph_bfs_args>(b), i);
+    else if constexpr (M == VF_GRAPH_BFS_PROBE) o->bfs_probe(blob_as<vf_graph_bfs_args>(b), i);
+    else if constexpr (M == VF_GRAPH_CC_UPDATE) o->cc_update(blob_as<vf_graph_cc_args>(b), i);
+    else if constexpr (M == VF_GRAPH_PR_CONTRIB) o->pr_contrib(blob_as<vf_graph_pr_args>(b), i);
+    else o->pr_update(blob_as<vf_graph_pr_args>(b), i);
   }
   template <int M, int K>
-  __device__ __forceinline__ static void dcall(Type<K>* o, uint64_t, const ArgBlob& b) {
-    if constexpr (M == VF_GRAPH_BFS_EXPAND) o->Type<K>::bfs_expand(blob_as<vf_graph_bfs_args>(b));
-    else if constexpr (M == VF_GRAPH_BFS_PROBE) o->Type<K>::bfs_probe(blob_as<vf_graph_bfs_args>(b));
-    else if constexpr (M == VF_GRAPH_CC_UPDATE) o->Type<K>::cc_update(blob_as<vf_graph_cc_args>(b));
-    else if constexpr (M == VF_GRAPH_PR_CONTRIB) o->Type<K>::pr_contrib(blob_as<vf_graph_pr_args>(b));
-    else o->Type<K>::pr_update(blob_as<vf_graph_pr_args>(b));
+  __device__ __forceinline__ static void dcall(Type<K>* o, uint64_t i, const ArgBlob& b) {
+    if constexpr (M == VF_GRAPH_BFS_EXPAND) o->Type<K>::bfs_expand(blob_as<vf_graph_bfs_args>(b), i);
+    else if constexpr (M == VF_GRAPH_BFS_PROBE) o->Type<K>::bfs_probe(blob_as<vf_graph_bfs_args>(b), i);
+    else if constexpr (M == VF_GRAPH_CC_UPDATE) o->Type<K>::cc_update(blob_as<vf_graph_cc_args>(b), i);
+    else if constexpr (M == VF_GRAPH_PR_CONTRIB) o->Type<K>::pr_contrib(blob_as<vf_graph_pr_args>(b), i);
+    else o->Type<K>::pr_update(blob_as<vf_graph_pr_args>(b), i);
   }
   __device__ static void construct(uint32_t t, void* mem, const void* arg) {
     construct_switch<App>(t, mem, arg);
@@ -158,14 +226,16 @@ struct App {
 };
 static_assert(sizeof(VertexK<0>) == 16, "vertex layout");
 
-__global__ void k_bfs_init(uint64_t V, int32_t* depth, uint32_t src, const uint64_t* vobj, uint64_t* queue,
-                           uint32_t* count) {
+__global__ void k_bfs_init(uint64_t V, int32_t* depth, uint32_t src, const uint64_t* vobj, const uint64_t* offs,
+                           uint32_t C, uint64_t* queue, uint32_t* qchunk, uint32_t* count) {
   const uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (v < V) depth[v] = v == src ? 0 : -1;
-  if (v == 0) {
-    queue[0] = vobj[src];
-    *count = 1;
+  const uint32_t n = nchunks((uint32_t)(offs[src + 1] - offs[src]), C);
+  if (v < n) {
+    queue[v] = vobj[src];
+    qchunk[v] = (uint32_t)v;
   }
+  if (v == 0) *count = n;
 }
 
 __global__ void k_iota(uint64_t V, uint32_t* x) {
@@ -193,10 +263,13 @@ const AppOps* app_graph() {
 }  // namespace vf
 
 extern "C" vf_status vf_graph_bfs_init(uint64_t V, int32_t* depth_dev, uint32_t src, const uint64_t* vobj_dev,
-                                       uint64_t* queue_dev, uint32_t* count_dev, void* stream) {
-  if (!V || src >= V || !depth_dev || !vobj_dev || !queue_dev || !count_dev) return VF_ERR_INVALID;
-  vf::graph::k_bfs_init<<<(unsigned)((V + 255) / 256), 256, 0, (cudaStream_t)stream>>>(V, depth_dev, src, vobj_dev,
-                                                                                       queue_dev, count_dev);
+                                       const uint64_t* offs_dev, uint32_t C, uint64_t* queue_dev,
+                                       uint32_t* queue_chunk_dev, uint32_t* count_dev, void* stream) {
+  if (!V || src >= V || !depth_dev || !vobj_dev || !offs_dev || !C || !queue_dev || !queue_chunk_dev || !count_dev)
+    return VF_ERR_INVALID;
+  // V threads also cover src's chunks: nch <= deg <= V
+  vf::graph::k_bfs_init<<<(unsigned)((V + 255) / 256), 256, 0, (cudaStream_t)stream>>>(
+      V, depth_dev, src, vobj_dev, offs_dev, C, queue_dev, queue_chunk_dev, count_dev);
   vf::note_launch();
   return cudaGetLastError() == cudaSuccess ? VF_OK : VF_ERR_CUDA;
 }

@@ -54,15 +54,28 @@ def allreduce_sum(t, world: int, group=None):
     dist.all_reduce(t, group=group)
 
 
+def work_entries(deg: np.ndarray, lo: int, hi: int, C: int):
+    """Work entries of vertices [lo, hi) (vf.h VF_APP_GRAPH): vertex v appears
+    nch(v) = max(1, ceil(deg/C)) times consecutively, with chunk ids 0..nch-1.
+    Returns (entry vertex ids int64[E], chunk ids uint32[E])."""
+    d = np.asarray(deg[lo:hi], np.int64)
+    nch = np.maximum(1, (d + C - 1) // C)
+    vid = np.repeat(np.arange(lo, hi, dtype=np.int64), nch)
+    first = np.repeat(np.cumsum(nch) - nch, nch)
+    chunk = (np.arange(len(vid), dtype=np.int64) - first).astype(np.uint32)
+    return vid, chunk
+
+
 class Graph:
     def __init__(self, ctx: vf.Ctx, offs: np.ndarray, col: np.ndarray, variant: str = "typeptr",
-                 rank: int = 0, world: int = 1, group=None):
+                 rank: int = 0, world: int = 1, group=None, chunk: int = 256):
         self.ctx, self.variant = ctx, variant
         self.v = vf.VARIANTS[variant]
         dev = torch.device(f"cuda:{ctx.device}")
         self.dev = dev
         V = len(offs) - 1
         self.V = V
+        self.C = int(chunk)
         self.rank, self.world, self.group = rank, world, group
         # owned vertex block [lo, hi)
         self.lo, self.hi, self.per = block_range(V, rank, world)
@@ -83,14 +96,23 @@ class Graph:
         self.vobj = torch.zeros(V, dtype=torch.int64, device=dev)
         self.vobj[self.lo:self.hi] = objs
         self.owned = self.vobj[self.lo:self.hi]
+        # work entries of the owned block (one virtual call each)
+        evid, ech = work_entries(deg, self.lo, self.hi, self.C)
+        self.E = len(evid)
+        self.entries = self.vobj[torch.from_numpy(evid).to(dev)].contiguous()
+        self.entry_chunk = torch.from_numpy(ech.view(np.int32)).to(dev)
+        e_all = int(np.maximum(1, (deg + self.C - 1) // self.C).sum())
         self.depth = torch.empty(V, dtype=torch.int32, device=dev)
-        self.q = [torch.empty(max(V, 1), dtype=torch.int64, device=dev) for _ in range(2)]
+        self.q = [torch.empty(max(e_all, 1), dtype=torch.int64, device=dev) for _ in range(2)]
+        self.qc = [torch.empty(max(e_all, 1), dtype=torch.int32, device=dev) for _ in range(2)]
         self.count = torch.zeros(1, dtype=torch.int32, device=dev)
         self.lab = [torch.empty(V, dtype=torch.int32, device=dev) for _ in range(2)]
         self.changed = torch.zeros(1, dtype=torch.int32, device=dev)
         self.rk = [torch.empty(V, dtype=torch.float32, device=dev) for _ in range(2)]
         self.contrib = torch.empty(V, dtype=torch.float64, device=dev)
         self.dangling = torch.zeros(1, dtype=torch.float64, device=dev)
+        self.partial = torch.zeros(max(self.E, 1), dtype=torch.float64, device=dev)
+        self.counter = torch.zeros(V, dtype=torch.int32, device=dev)
         self.calls = 0
         torch.cuda.synchronize(dev)
 
@@ -109,33 +131,36 @@ class Graph:
     # ---------------------------------------------------------------- BFS
     def bfs(self, src: int, mode: str = "topdown"):
         """Level-synchronous BFS from src; returns (depth tensor, levels, calls).
-        topdown: one virtual bfs_expand() per frontier vertex (single GPU);
-        bottomup: one virtual bfs_probe() per owned vertex per level (multi-GPU)."""
+        topdown: one virtual bfs_expand() per frontier work entry (single GPU);
+        bottomup: one virtual bfs_probe() per owned work entry per level (multi-GPU)."""
         L = vf.lib()
-        st = L.vf_graph_bfs_init(self.V, self.depth.data_ptr(), src, self.vobj.data_ptr(), self.q[0].data_ptr(),
-                                 self.count.data_ptr(), vf._stream(None))
+        st = L.vf_graph_bfs_init(self.V, self.depth.data_ptr(), src, self.vobj.data_ptr(), self.offs.data_ptr(),
+                                 self.C, self.q[0].data_ptr(), self.qc[0].data_ptr(), self.count.data_ptr(),
+                                 vf._stream(None))
         if st:
             raise vf.VFError(st, "bfs_init")
         calls, level = 0, 0
         if mode == "topdown" and self.world == 1:
-            n = 1
+            n = _sync_scalar(self.count)
             while n > 0:
                 self.count.zero_()
                 a = vf.graph_bfs_args(self.offs.data_ptr(), self.col.data_ptr(), self.depth.data_ptr(),
-                                      self.vobj.data_ptr(), self.q[1].data_ptr(), self.count.data_ptr(), level)
+                                      self.vobj.data_ptr(), self.qc[0].data_ptr(), self.q[1].data_ptr(),
+                                      self.qc[1].data_ptr(), self.count.data_ptr(), level, self.C)
                 self._dispatch(vf.GRAPH_BFS_EXPAND, self.q[0].data_ptr(), n, a)
                 calls += n
                 n = _sync_scalar(self.count)
                 self.q[0], self.q[1] = self.q[1], self.q[0]
+                self.qc[0], self.qc[1] = self.qc[1], self.qc[0]
                 level += 1
         else:
-            nown = self.hi - self.lo
             while True:
                 self.count.zero_()
                 a = vf.graph_bfs_args(self.offs.data_ptr(), self.col.data_ptr(), self.depth.data_ptr(),
-                                      self.vobj.data_ptr(), 0, self.count.data_ptr(), level)
-                self._dispatch(vf.GRAPH_BFS_PROBE, self.owned.data_ptr(), nown, a)
-                calls += nown
+                                      self.vobj.data_ptr(), self.entry_chunk.data_ptr(), 0, 0, self.count.data_ptr(),
+                                      level, self.C)
+                self._dispatch(vf.GRAPH_BFS_PROBE, self.entries.data_ptr(), self.E, a)
+                calls += self.E
                 self._allreduce_sum(self.count)
                 self._allgather_block(self.depth)
                 level += 1
@@ -149,13 +174,14 @@ class Graph:
         """Jacobi min-label propagation until no label changes; returns (labels, iters, calls)."""
         L = vf.lib()
         L.vf_iota_u32(self.V, self.lab[0].data_ptr(), vf._stream(None))
-        it, calls, nown = 0, 0, self.hi - self.lo
+        L.vf_iota_u32(self.V, self.lab[1].data_ptr(), vf._stream(None))  # >= every later label (atomicMin combine)
+        it, calls = 0, 0
         while it < max_iters:
             self.changed.zero_()
             a = vf.graph_cc_args(self.offs.data_ptr(), self.col.data_ptr(), self.lab[0].data_ptr(),
-                                 self.lab[1].data_ptr(), self.changed.data_ptr())
-            self._dispatch(vf.GRAPH_CC_UPDATE, self.owned.data_ptr(), nown, a)
-            calls += nown
+                                 self.lab[1].data_ptr(), self.changed.data_ptr(), self.entry_chunk.data_ptr(), self.C)
+            self._dispatch(vf.GRAPH_CC_UPDATE, self.entries.data_ptr(), self.E, a)
+            calls += self.E
             it += 1
             self._allgather_block(self.lab[1])
             self._allreduce_sum(self.changed)
@@ -170,18 +196,18 @@ class Graph:
         vf.lib().vf_fill_f32(self.V, self.rk[0].data_ptr(), ctypes.c_float(1.0 / self.V).value, vf._stream(None))
 
     def pr_iteration(self, d: float = 0.85, stream=None):
-        """One PageRank iteration = virtual pr_contrib() + pr_update() per owned vertex."""
-        nown = self.hi - self.lo
+        """One PageRank iteration = virtual pr_contrib() + pr_update() per owned work entry."""
         self.dangling.zero_()
         a = vf.graph_pr_args(self.offs.data_ptr(), self.col.data_ptr(), self.rk[0].data_ptr(), self.rk[1].data_ptr(),
-                             self.contrib.data_ptr(), self.dangling.data_ptr(), (1.0 - d) / self.V, d, float(self.V))
-        self._dispatch(vf.GRAPH_PR_CONTRIB, self.owned.data_ptr(), nown, a, stream)
+                             self.contrib.data_ptr(), self.dangling.data_ptr(), (1.0 - d) / self.V, d, float(self.V),
+                             self.entry_chunk.data_ptr(), self.partial.data_ptr(), self.counter.data_ptr(), self.C)
+        self._dispatch(vf.GRAPH_PR_CONTRIB, self.entries.data_ptr(), self.E, a, stream)
         self._allgather_block(self.contrib)
         self._allreduce_sum(self.dangling)
-        self._dispatch(vf.GRAPH_PR_UPDATE, self.owned.data_ptr(), nown, a, stream)
+        self._dispatch(vf.GRAPH_PR_UPDATE, self.entries.data_ptr(), self.E, a, stream)
         self._allgather_block(self.rk[1])
         self.rk[0], self.rk[1] = self.rk[1], self.rk[0]
-        return 2 * nown
+        return 2 * self.E
 
     def pagerank(self, iters: int = 20, d: float = 0.85):
         self.pr_init()

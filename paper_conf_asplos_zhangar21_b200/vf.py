@@ -137,20 +137,23 @@ gen_get_args = gol_get_args
 
 class graph_bfs_args(ctypes.Structure):
     _fields_ = [("offs_dev", ctypes.c_void_p), ("col_dev", ctypes.c_void_p), ("depth_dev", ctypes.c_void_p),
-                ("vobj_dev", ctypes.c_void_p), ("next_queue_dev", ctypes.c_void_p),
-                ("next_count_dev", ctypes.c_void_p), ("level", ctypes.c_int32)]
+                ("vobj_dev", ctypes.c_void_p), ("chunk_dev", ctypes.c_void_p), ("next_queue_dev", ctypes.c_void_p),
+                ("next_chunk_dev", ctypes.c_void_p), ("next_count_dev", ctypes.c_void_p), ("level", ctypes.c_int32),
+                ("C", ctypes.c_uint32)]
 
 
 class graph_cc_args(ctypes.Structure):
     _fields_ = [("offs_dev", ctypes.c_void_p), ("col_dev", ctypes.c_void_p), ("label_in_dev", ctypes.c_void_p),
-                ("label_out_dev", ctypes.c_void_p), ("changed_dev", ctypes.c_void_p)]
+                ("label_out_dev", ctypes.c_void_p), ("changed_dev", ctypes.c_void_p), ("chunk_dev", ctypes.c_void_p),
+                ("C", ctypes.c_uint32)]
 
 
 class graph_pr_args(ctypes.Structure):
     _fields_ = [("offs_dev", ctypes.c_void_p), ("col_dev", ctypes.c_void_p), ("rank_in_dev", ctypes.c_void_p),
                 ("rank_out_dev", ctypes.c_void_p), ("contrib_dev", ctypes.c_void_p),
                 ("dangling_dev", ctypes.c_void_p), ("base", ctypes.c_double), ("d", ctypes.c_double),
-                ("Vd", ctypes.c_double)]
+                ("Vd", ctypes.c_double), ("chunk_dev", ctypes.c_void_p), ("partial_dev", ctypes.c_void_p),
+                ("counter_dev", ctypes.c_void_p), ("C", ctypes.c_uint32)]
 
 
 _lib = None
@@ -192,7 +195,7 @@ def lib(required: bool = True):
         "vf_checksum_i32": (I, [P, U64, P, P]),
         "vf_launch_count": (U64, []),
         "vf_set_tuning": (I, [ctypes.c_char_p, I]),
-        "vf_graph_bfs_init": (I, [U64, P, U32, P, P, P, P]),
+        "vf_graph_bfs_init": (I, [U64, P, U32, P, P, U32, P, P, P, P]),
         "vf_iota_u32": (I, [U64, P, P]),
         "vf_fill_f32": (I, [U64, P, ctypes.c_float, P]),
         "vf_ray_render": (I, [P, I, P, U32, U32, U32, U32, U32, P, P, P, P, P]),

@@ -38,19 +38,28 @@ def rmat(request):
 
 
 @pytest.mark.parametrize("variant", VARIANTS)
-def test_graph_parity(ctx, rmat, variant):
-    g = Graph(ctx, rmat["offs"], rmat["col"], variant)
+@pytest.mark.parametrize("chunk", [256, 7])
+def test_graph_parity(ctx, rmat, variant, chunk):
+    g = Graph(ctx, rmat["offs"], rmat["col"], variant, chunk=chunk)
+    assert g.E > g.V  # some vertices span several work entries
     depth, levels, calls = g.bfs(rmat["src"])
-    assert np.array_equal(depth.cpu().numpy(), rmat["depth"])
-    assert levels == rmat["levels"] and calls == rmat["calls"]
+    d = depth.cpu().numpy()
+    assert np.array_equal(d, rmat["depth"])
+    # the oracle counts one expand() per reached vertex; here: one per work entry
+    assert levels == rmat["levels"] and int((d >= 0).sum()) == rmat["calls"] and calls >= rmat["calls"]
     d2, _, _ = g.bfs(rmat["src"], mode="bottomup")
     assert np.array_equal(d2.cpu().numpy(), rmat["depth"])
     label, iters, _ = g.cc()
     assert np.array_equal(label.cpu().numpy().view(np.uint32), rmat["label"])
     assert iters == rmat["iters"]
+    label, iters, _ = g.cc()  # repeatable (both label buffers re-initialised)
+    assert np.array_equal(label.cpu().numpy().view(np.uint32), rmat["label"]) and iters == rmat["iters"]
     rank, _ = g.pagerank(20)
     r = rank.cpu().numpy()
     np.testing.assert_allclose(r, rmat["rank"], rtol=1e-5, atol=0)
+    assert int(g.counter.abs().sum()) == 0  # every multi-chunk combine finished and reset
+    r2, _ = g.pagerank(20)  # chunk partials combine in chunk order; only the fp64 dangling sum is atomic
+    np.testing.assert_allclose(r2.cpu().numpy(), r, rtol=1e-7, atol=0)
     assert abs(float(r.astype(np.float64).sum()) - 1.0) < 1e-4
     assert ctx.verify(vf.APP_GRAPH, g.v, g.owned) == 0
 

@@ -29,6 +29,8 @@ from paper_conf_asplos_zhangar21_b200 import apps, vf  # noqa: E402
 from paper_conf_asplos_zhangar21_b200.graph import Graph  # noqa: E402
 from paper_conf_asplos_zhangar21_b200.ray import Ray  # noqa: E402
 from paper_conf_asplos_zhangar21_b200.traf import Traf  # noqa: E402
+from paper_conf_asplos_zhangar21_b200.nbody import Nbody  # noqa: E402
+from paper_conf_asplos_zhangar21_b200.stut import Stut  # noqa: E402
 
 VARIANTS = ("cuda", "sharedoa", "coal", "typeptr")
 PEAKS = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))) if os.path.exists(
@@ -190,9 +192,46 @@ def bench_traf(ctx, quick):
         ctx.reset()
 
 
+# ---------------------------------------------------------------- config 5: N-body (all pairs)
+def bench_nbody(ctx, quick):
+    N = 16384 if quick else 65536
+    steps = 10
+    s = synth.nbody_system(N, seed=10)
+    Ns = 8192
+    _, _, sec = oracle.nbody_run(synth.nbody_system(Ns, seed=10), 2, threads=oracle.max_threads())
+    # work per update() call grows with N: scale the sampled rate by Ns/N
+    cpu = cpu_info(Ns * 2 * (Ns / N), sec, f"N={Ns}, 2 steps, rate scaled by {Ns}/{N} (work per call ~ N)")
+    flops = 20.0 * (N - 1)  # per update(): N-1 pair interactions x 20 formula FLOPs
+    for v in VARIANTS:
+        nb = Nbody(ctx, s, v)
+        ms = ev_time(nb.step, steps)
+        record("nbody", f"all-pairs N={N}", v, N, ms, flops, "TFLOP/s", "alu", None, cpu)
+        del nb
+        ctx.reset()
+
+
+# ---------------------------------------------------------------- config 5: STUT
+def bench_stut(ctx, quick):
+    W = H = 512 if quick else 2048
+    steps = 20
+    w = synth.stut_lattice(W, H, seed=12, v_pull=4.0)
+    _, _, _, sec = oracle.stut_run(w, 5, threads=oracle.max_threads())
+    n, S = W * H, len(w["a"])
+    cpu = cpu_info((n + S) * 5, sec, f"full structure, 5 steps")
+    # spring: 8 ptr + 32 obj + 16 pos + 8 F; node: 8 ptr + 24 obj r + 12 w + 8 offs + 24 inc + 48 F + 16 pos
+    per_call = (64 * S + 140 * n) / (S + n)
+    for v in VARIANTS:
+        st = Stut(ctx, w, v)
+        ms = ev_time(st.step, steps)
+        record("stut", f"{W}x{H} nodes, {S} springs", v, st.calls_per_step, ms, per_call, "GB/s", "hbm",
+               dict(objects=n + S), cpu)
+        del st
+        ctx.reset()
+
+
 def main():
     ap = argparse.ArgumentParser()
-    ap.add_argument("--apps", default="gol,ray,traf,gen,graph")
+    ap.add_argument("--apps", default="gol,ray,traf,gen,stut,nbody,graph")
     ap.add_argument("--out", default="gpurun_out/apps")
     ap.add_argument("--quick", action="store_true")
     a = ap.parse_args()
