@@ -391,6 +391,20 @@ vf_status vf_gen_swap(vf_ctx* ctx, uint64_t ncells, const uint8_t* state_prev_de
                       const uint8_t* state_next_dev, uint64_t* grid_dev, const uint64_t* dead_dev,
                       const uint64_t* alive_dev, const uint64_t* dying_dev, void* stream);
 
+/* Fused generation (B200 design): steps (1) neighbours, (2) one
+ * virtual next() per cell under variant v, (3) swap, done per cell by ONE
+ * thread in ONE launch — identical results to vf_gol_neighbors + vf_dispatch
+ * (VF_GOL_NEXT, args {nbr_dev, next_dev}) + vf_gol_swap. grid_dev[c] must be
+ * cell c's current object (its own cell field = c). */
+vf_status vf_gol_step(vf_ctx* ctx, vf_variant v, uint32_t W, uint32_t H, int torus, const uint8_t* state_prev_dev,
+                      uint8_t* state_next_dev, uint8_t* nbr_dev, uint64_t* grid_dev, const uint64_t* alive_dev,
+                      const uint64_t* dead_dev, void* stream);
+/* Same for GEN (VF_GEN_NEXT with {nbr, next, born_mask, survive_mask, C}, then vf_gen_swap). */
+vf_status vf_gen_step(vf_ctx* ctx, vf_variant v, uint32_t W, uint32_t H, int torus, const uint8_t* state_prev_dev,
+                      uint8_t* state_next_dev, uint8_t* nbr_dev, uint64_t* grid_dev, const uint64_t* dead_dev,
+                      const uint64_t* alive_dev, const uint64_t* dying_dev, uint32_t born_mask,
+                      uint32_t survive_mask, uint32_t C, void* stream);
+
 /* Config 3 ray tracer (readings G24, G25): render rows [row0, row0+nrows) of
  * a W x H image over S shapes of VF_APP_RAY (type ids 0 Plane, 1 Sphere,
  * 2 Rect, 3 Triangle; constructor argument = 12 fp32 params, see

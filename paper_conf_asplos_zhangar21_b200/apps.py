@@ -93,11 +93,17 @@ class Gol:
         self.parity = 0
         torch.cuda.synchronize(dev)
 
-    def gen(self, stream=None):
+    def gen(self, stream=None, fused: bool = True):
+        """One generation. fused (default, B200 design): one vf_gol_step launch;
+        else the three phases as separate calls (neighbours, dispatch, swap)."""
         cur, nxt = (self.state, self.next) if self.parity == 0 else (self.next, self.state)
-        vf.gol_neighbors(self.W, self.H, cur, self.nbr, self.torus, stream)
-        self.ctx.dispatch(self.v, vf.APP_GOL, vf.GOL_NEXT, self.grid, self.args[self.parity], stream=stream)
-        vf.gol_swap(self.ctx, cur, nxt, self.grid, self.alive, self.dead, stream)
+        if fused:
+            vf.gol_step(self.ctx, self.v, self.W, self.H, self.torus, cur, nxt, self.nbr, self.grid, self.alive,
+                        self.dead, stream)
+        else:
+            vf.gol_neighbors(self.W, self.H, cur, self.nbr, self.torus, stream)
+            self.ctx.dispatch(self.v, vf.APP_GOL, vf.GOL_NEXT, self.grid, self.args[self.parity], stream=stream)
+            vf.gol_swap(self.ctx, cur, nxt, self.grid, self.alive, self.dead, stream)
         self.parity ^= 1
 
     @property
@@ -144,16 +150,21 @@ class Gen:
         self.next = torch.empty_like(self.state)
         self.nbr = torch.empty_like(self.state)
         bm, sm = rule_masks(born, survive)
+        self.rule = (bm, sm, C)
         self.args = [vf.gen_next_args(self.nbr.data_ptr(), self.next.data_ptr(), bm, sm, C),
                      vf.gen_next_args(self.nbr.data_ptr(), self.state.data_ptr(), bm, sm, C)]
         self.parity = 0
         torch.cuda.synchronize(dev)
 
-    def gen(self, stream=None):
+    def gen(self, stream=None, fused: bool = True):
         cur, nxt = (self.state, self.next) if self.parity == 0 else (self.next, self.state)
-        vf.gol_neighbors(self.W, self.H, cur, self.nbr, self.torus, stream)
-        self.ctx.dispatch(self.v, vf.APP_GEN, vf.GEN_NEXT, self.grid, self.args[self.parity], stream=stream)
-        vf.gen_swap(self.ctx, cur, nxt, self.grid, self.dead, self.alive, self.dying, stream)
+        if fused:
+            vf.gen_step(self.ctx, self.v, self.W, self.H, self.torus, cur, nxt, self.nbr, self.grid, self.dead,
+                        self.alive, self.dying, *self.rule, stream)
+        else:
+            vf.gol_neighbors(self.W, self.H, cur, self.nbr, self.torus, stream)
+            self.ctx.dispatch(self.v, vf.APP_GEN, vf.GEN_NEXT, self.grid, self.args[self.parity], stream=stream)
+            vf.gen_swap(self.ctx, cur, nxt, self.grid, self.dead, self.alive, self.dying, stream)
         self.parity ^= 1
 
     @property

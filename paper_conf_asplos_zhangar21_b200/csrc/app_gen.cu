@@ -6,6 +6,8 @@
 // change is a pointer swap (k_gen_swap), exactly as in app_gol.cu.
 //
 // Object layout (16 B): { vTable* (8 B), u32 cell, u16 counter, u8 stage, u8 pad }.
+#include <cstring>
+
 #include "dispatch.cuh"
 
 namespace vf {
@@ -122,7 +124,43 @@ __global__ void k_gen_swap(uint64_t n, const uint8_t* __restrict__ prev, const u
   }
 }
 
+// Fused generation (vf_gen_step): neighbours -> virtual next() -> swap per cell.
+struct Step {
+  uint32_t W, H;
+  int torus;
+  const uint8_t* prev;
+  const uint8_t* next;
+  uint8_t* nbr;
+  uint64_t* grid;
+  const uint64_t* dead;
+  const uint64_t* alive;
+  const uint64_t* dying;
+  __device__ __forceinline__ void pre(uint64_t c) const { nbr[c] = count_live(W, H, torus, prev, c); }
+  __device__ __forceinline__ uint64_t ptr(uint64_t c) const { return grid[c]; }
+  __device__ __forceinline__ void post(uint64_t c) const {
+    const uint8_t s = next[c];
+    const int k = kind(s);
+    if (k != kind(prev[c])) {
+      const uint64_t p = k == 0 ? dead[c] : k == 1 ? alive[c] : dying[c];
+      grid[c] = p;
+      Cell* o = reinterpret_cast<Cell*>(strip(p));
+      o->counter = 0;
+      if (k == 2) o->stage = s;
+    }
+  }
+};
+
 }  // namespace gen
+
+cudaError_t gen_step(int variant, uint32_t W, uint32_t H, int torus, const uint8_t* prev, uint8_t* next, uint8_t* nbr,
+                     uint64_t* grid, const uint64_t* dead, const uint64_t* alive, const uint64_t* dying,
+                     uint32_t born, uint32_t survive, uint32_t C, const DevTable& tbl, cudaStream_t s) {
+  vf_gen_next_args a{nbr, next, born, survive, C};
+  ArgBlob blob{};
+  memcpy(blob.b, &a, sizeof a);
+  const gen::Step st{W, H, torus, prev, next, nbr, grid, dead, alive, dying};
+  return launch_step<gen::App, VF_GEN_NEXT>(variant, (uint64_t)W * H, blob, tbl, st, s);
+}
 
 static const uint32_t kGenBytes[3] = {16, 16, 16};
 static const uint32_t kGenArgs[2] = {sizeof(vf_gen_next_args), sizeof(vf_gen_get_args)};

@@ -7,6 +7,8 @@
 // Object layout (16 B): { vTable* (8 B), u32 cell, u16 counter, u16 pad }.
 // counter = age (Alive) / dead_for (Dead): incremented by next(), reset to 0
 // when the cell switches to this object.
+#include <cstring>
+
 #include "dispatch.cuh"
 
 namespace vf {
@@ -86,23 +88,7 @@ __global__ void k_neighbors(uint32_t W, uint32_t H, int torus, const uint8_t* __
                             uint8_t* __restrict__ nb) {
   const uint64_t c = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (c >= (uint64_t)W * H) return;
-  const int y = (int)(c / W), x = (int)(c % W);
-  int n = 0;
-#pragma unroll
-  for (int dy = -1; dy <= 1; ++dy)
-#pragma unroll
-    for (int dx = -1; dx <= 1; ++dx) {
-      if (dx == 0 && dy == 0) continue;
-      int yy = y + dy, xx = x + dx;
-      if (torus) {
-        yy = (yy + (int)H) % (int)H;
-        xx = (xx + (int)W) % (int)W;
-      } else if (yy < 0 || yy >= (int)H || xx < 0 || xx >= (int)W) {
-        continue;
-      }
-      n += st[(uint64_t)yy * W + xx] == 1;
-    }
-  nb[c] = (uint8_t)n;
+  nb[c] = count_live(W, H, torus, st, c);
 }
 
 __global__ void k_swap(uint64_t n, const uint8_t* __restrict__ prev, const uint8_t* __restrict__ next,
@@ -118,7 +104,39 @@ __global__ void k_swap(uint64_t n, const uint8_t* __restrict__ prev, const uint8
   }
 }
 
+// Fused generation (vf_gol_step): neighbours -> virtual next() -> swap per cell.
+struct Step {
+  uint32_t W, H;
+  int torus;
+  const uint8_t* prev;
+  const uint8_t* next;
+  uint8_t* nbr;
+  uint64_t* grid;
+  const uint64_t* alive;
+  const uint64_t* dead;
+  __device__ __forceinline__ void pre(uint64_t c) const { nbr[c] = count_live(W, H, torus, prev, c); }
+  __device__ __forceinline__ uint64_t ptr(uint64_t c) const { return grid[c]; }
+  __device__ __forceinline__ void post(uint64_t c) const {
+    const uint8_t s = next[c];
+    if (s != prev[c]) {
+      const uint64_t p = s ? alive[c] : dead[c];
+      grid[c] = p;
+      reinterpret_cast<Cell*>(strip(p))->counter = 0;
+    }
+  }
+};
+
 }  // namespace gol
+
+cudaError_t gol_step(int variant, uint32_t W, uint32_t H, int torus, const uint8_t* prev, uint8_t* next, uint8_t* nbr,
+                     uint64_t* grid, const uint64_t* alive, const uint64_t* dead, const DevTable& tbl,
+                     cudaStream_t s) {
+  vf_gol_next_args a{nbr, next};
+  ArgBlob blob{};
+  memcpy(blob.b, &a, sizeof a);
+  const gol::Step st{W, H, torus, prev, next, nbr, grid, alive, dead};
+  return launch_step<gol::App, VF_GOL_NEXT>(variant, (uint64_t)W * H, blob, tbl, st, s);
+}
 
 static const uint32_t kGolBytes[2] = {16, 16};
 static const uint32_t kGolArgs[2] = {sizeof(vf_gol_next_args), sizeof(vf_gol_get_args)};

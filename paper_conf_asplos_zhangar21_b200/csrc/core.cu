@@ -727,6 +727,40 @@ vf_status vf_ray_render(vf_ctx* c, vf_variant v, const uint64_t* shapes_dev, uin
   return VF_OK;
 }
 
+vf_status vf_gol_step(vf_ctx* c, vf_variant v, uint32_t W, uint32_t H, int torus, const uint8_t* prev_dev,
+                      uint8_t* next_dev, uint8_t* nbr_dev, uint64_t* grid_dev, const uint64_t* alive_dev,
+                      const uint64_t* dead_dev, void* stream) {
+  vf_status st = check_app(c, VF_APP_GOL);
+  if (st) return st;
+  if ((unsigned)v > VF_TYPEPTR) return fail(c, VF_ERR_INVALID, "variant %d", (int)v);
+  if ((uint64_t)W * H && (!prev_dev || !next_dev || !nbr_dev || !grid_dev || !alive_dev || !dead_dev))
+    return fail(c, VF_ERR_INVALID, "gol_step arguments");
+  if ((st = set_device(c)) || (st = ensure_vptrs(c, VF_APP_GOL))) return st;
+  if (v == VF_COAL && c->tables[VF_APP_GOL].K > VF_MAX_RANGES)
+    return fail(c, VF_ERR_TABLE_FULL, "K = %u > %u", c->tables[VF_APP_GOL].K, VF_MAX_RANGES);
+  CUDA_TRY(c, gol_step((int)v, W, H, torus, prev_dev, next_dev, nbr_dev, grid_dev, alive_dev, dead_dev,
+                       dev_table(c, VF_APP_GOL), reinterpret_cast<cudaStream_t>(stream)));
+  return VF_OK;
+}
+
+vf_status vf_gen_step(vf_ctx* c, vf_variant v, uint32_t W, uint32_t H, int torus, const uint8_t* prev_dev,
+                      uint8_t* next_dev, uint8_t* nbr_dev, uint64_t* grid_dev, const uint64_t* dead_dev,
+                      const uint64_t* alive_dev, const uint64_t* dying_dev, uint32_t born_mask,
+                      uint32_t survive_mask, uint32_t C, void* stream) {
+  vf_status st = check_app(c, VF_APP_GEN);
+  if (st) return st;
+  if ((unsigned)v > VF_TYPEPTR) return fail(c, VF_ERR_INVALID, "variant %d", (int)v);
+  if ((uint64_t)W * H && (!prev_dev || !next_dev || !nbr_dev || !grid_dev || !dead_dev || !alive_dev || !dying_dev))
+    return fail(c, VF_ERR_INVALID, "gen_step arguments");
+  if (C < 2 || C > 255) return fail(c, VF_ERR_INVALID, "C = %u", C);
+  if ((st = set_device(c)) || (st = ensure_vptrs(c, VF_APP_GEN))) return st;
+  if (v == VF_COAL && c->tables[VF_APP_GEN].K > VF_MAX_RANGES)
+    return fail(c, VF_ERR_TABLE_FULL, "K = %u > %u", c->tables[VF_APP_GEN].K, VF_MAX_RANGES);
+  CUDA_TRY(c, gen_step((int)v, W, H, torus, prev_dev, next_dev, nbr_dev, grid_dev, dead_dev, alive_dev, dying_dev,
+                       born_mask, survive_mask, C, dev_table(c, VF_APP_GEN), reinterpret_cast<cudaStream_t>(stream)));
+  return VF_OK;
+}
+
 vf_status vf_dispatch_cuda(vf_ctx* c, uint32_t app, uint32_t m, const uint64_t* o, uint64_t n,
                            const void* a, size_t ab, void* s) {
   return vf_dispatch(c, VF_CUDA, app, m, o, n, a, ab, s);

@@ -857,6 +857,106 @@ cudaError_t verify_impl(int variant, const uint64_t* ptrs, uint64_t n, unsigned 
   return cudaGetLastError();
 }
 
+// ---------------------------------------------------------------------------
+// Fused per-index step (B200 design for apps whose step is a non-virtual
+// pre-phase, the virtual call and a non-virtual post-phase on the same index,
+// e.g. the cellular automata): one thread per index runs all three, so a
+// whole step is ONE launch and the pre-phase's result reaches the method
+// through L1 instead of a separate kernel round trip. The call itself is the
+// variant's: a plain virtual call (CUDA / SharedOA) or resolve + warp-grouped
+// direct call (COAL / TypePointer). Step provides
+//   __device__ void pre(uint64_t c) const; uint64_t ptr(uint64_t c) const;
+//   void post(uint64_t c) const;
+// ---------------------------------------------------------------------------
+template <class App, int M, class R, class Step>
+__global__ void __launch_bounds__(kBlock) k_step_grouped(uint64_t n, ArgBlob args, DevTable tbl, Step st) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  if constexpr (R::kNeedsTable) R::stage(smem, tbl);
+  uint32_t hint = 0;
+  // CTA-uniform loop: every lane of every warp iterates together (full-mask collectives)
+  for (uint64_t base = (uint64_t)blockIdx.x * kBlock; base < n; base += (uint64_t)gridDim.x * kBlock) {
+    const uint64_t c = base + threadIdx.x;
+    const bool valid = c < n;
+    uint64_t p = 0, a = 0;
+    uint32_t t = kNF;
+    if (valid) {
+      st.pre(c);
+      p = st.ptr(c);
+    }
+    if (p) t = R::resolve(smem, tbl.P, p, a, hint);
+    group_call<App, M>(t, a, p, c, args, tbl);
+    if (valid) st.post(c);
+  }
+}
+
+template <class App, int M, class Step>
+__global__ void __launch_bounds__(kBlock) k_step_virtual(uint64_t n, ArgBlob args, Step st) {
+  const uint64_t c = (uint64_t)blockIdx.x * kBlock + threadIdx.x;
+  if (c >= n) return;
+  st.pre(c);
+  const uint64_t p = st.ptr(c);
+  if (p) App::template vcall<M>(reinterpret_cast<typename App::Base*>(p), c, args);
+  st.post(c);
+}
+
+template <class App, int M, class R, class Step>
+cudaError_t launch_step_grouped(uint64_t n, const ArgBlob& args, const DevTable& tbl, const Step& st,
+                                cudaStream_t s) {
+  auto kern = k_step_grouped<App, M, R, Step>;
+  const size_t sm = R::kNeedsTable ? table_smem(tbl) : 0;
+  static int occ = -1;
+  static size_t occ_sm = ~(size_t)0;
+  if (occ < 0 || occ_sm != sm) {
+    if (sm > 48 * 1024) cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kBlock, sm);
+    if (occ < 1) occ = 1;
+    occ_sm = sm;
+  }
+  kern<<<grid_for(n, kBlock, (uint64_t)num_sms() * occ), kBlock, sm, s>>>(n, args, tbl, st);
+  note_launch();
+  return cudaGetLastError();
+}
+
+template <class App, int M, class Step>
+cudaError_t launch_step(int variant, uint64_t n, const ArgBlob& args, const DevTable& tbl, const Step& st,
+                        cudaStream_t s) {
+  if (n == 0) return cudaSuccess;
+  switch (variant) {
+    case VF_CUDA:
+    case VF_SHAREDOA:
+      k_step_virtual<App, M, Step><<<grid_for(n, kBlock, ~0u), kBlock, 0, s>>>(n, args, st);
+      note_launch();
+      return cudaGetLastError();
+    case VF_COAL:
+      return launch_step_grouped<App, M, ResolveCOAL, Step>(n, args, tbl, st, s);
+    case VF_TYPEPTR:
+      return launch_step_grouped<App, M, ResolveTP, Step>(n, args, tbl, st, s);
+  }
+  return cudaErrorInvalidValue;
+}
+
+// live (state == 1) neighbours of cell c of a W x H grid (dead border, or torus)
+__device__ __forceinline__ uint8_t count_live(uint32_t W, uint32_t H, int torus, const uint8_t* __restrict__ st,
+                                              uint64_t c) {
+  const int y = (int)(c / W), x = (int)(c % W);
+  int n = 0;
+#pragma unroll
+  for (int dy = -1; dy <= 1; ++dy)
+#pragma unroll
+    for (int dx = -1; dx <= 1; ++dx) {
+      if (dx == 0 && dy == 0) continue;
+      int yy = y + dy, xx = x + dx;
+      if (torus) {
+        yy = (yy + (int)H) % (int)H;
+        xx = (xx + (int)W) % (int)W;
+      } else if (yy < 0 || yy >= (int)H || xx < 0 || xx >= (int)W) {
+        continue;
+      }
+      n += st[(uint64_t)yy * W + xx] == 1;
+    }
+  return (uint8_t)n;
+}
+
 // construct-by-type helpers for apps
 template <class App, int K = 0>
 __device__ __forceinline__ void construct_switch(uint32_t t, void* mem, const void* arg) {

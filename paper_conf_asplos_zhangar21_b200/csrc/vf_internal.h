@@ -71,6 +71,14 @@ cudaError_t ray_render(int variant, const uint64_t* objs, uint32_t S, uint32_t W
                        uint32_t nrows, const float* cam5, const float* albedo12, float* rgb, int32_t* hid,
                        const DevTable& tbl, cudaStream_t s);
 
+// fused cellular-automaton generations (app_gol.cu / app_gen.cu)
+cudaError_t gol_step(int variant, uint32_t W, uint32_t H, int torus, const uint8_t* prev, uint8_t* next, uint8_t* nbr,
+                     uint64_t* grid, const uint64_t* alive, const uint64_t* dead, const DevTable& tbl,
+                     cudaStream_t s);
+cudaError_t gen_step(int variant, uint32_t W, uint32_t H, int torus, const uint8_t* prev, uint8_t* next, uint8_t* nbr,
+                     uint64_t* grid, const uint64_t* dead, const uint64_t* alive, const uint64_t* dying,
+                     uint32_t born, uint32_t survive, uint32_t C, const DevTable& tbl, cudaStream_t s);
+
 // Benchmark / ablation knobs set through vf_set_tuning (-1 = app default).
 struct Tuning {
   int unroll = -1;    // objects per thread in the grouped kernels (1, 2, 4)

@@ -38,7 +38,7 @@ SYMBOLS = [
     "vf_regions", "vf_type_vptrs", "vf_resolve", "vf_verify_types", "vf_dispatch_cuda",
     "vf_dispatch_sharedoa", "vf_dispatch_coal", "vf_dispatch_typeptr", "vf_dispatch",
     "vf_gol_neighbors", "vf_gol_swap", "vf_gen_swap", "vf_checksum_i32", "vf_launch_count", "vf_set_tuning",
-    "vf_graph_bfs_init", "vf_iota_u32", "vf_fill_f32", "vf_ray_render",
+    "vf_graph_bfs_init", "vf_iota_u32", "vf_fill_f32", "vf_ray_render", "vf_gol_step", "vf_gen_step",
 ]
 APP_RAY = 4
 APP_TRAF = 5
@@ -199,6 +199,8 @@ def lib(required: bool = True):
         "vf_iota_u32": (I, [U64, P, P]),
         "vf_fill_f32": (I, [U64, P, ctypes.c_float, P]),
         "vf_ray_render": (I, [P, I, P, U32, U32, U32, U32, U32, P, P, P, P, P]),
+        "vf_gol_step": (I, [P, I, U32, U32, I, P, P, P, P, P, P, P]),
+        "vf_gen_step": (I, [P, I, U32, U32, I, P, P, P, P, P, P, P, U32, U32, U32, P]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)
@@ -389,6 +391,21 @@ def gen_swap(ctx: Ctx, prev, nxt, grid, dead, alive, dying, stream=None):
                            _ptr(alive), _ptr(dying), _stream(stream))
     if st:
         raise VFError(st, "gen_swap")
+
+
+def gol_step(ctx: Ctx, variant: int, W, H, torus, prev, nxt, nbr, grid, alive, dead, stream=None):
+    st = lib().vf_gol_step(ctx.h, variant, W, H, int(torus), _ptr(prev), _ptr(nxt), _ptr(nbr), _ptr(grid),
+                           _ptr(alive), _ptr(dead), _stream(stream))
+    if st:
+        ctx._check(st, "gol_step")
+
+
+def gen_step(ctx: Ctx, variant: int, W, H, torus, prev, nxt, nbr, grid, dead, alive, dying, born, survive, C,
+             stream=None):
+    st = lib().vf_gen_step(ctx.h, variant, W, H, int(torus), _ptr(prev), _ptr(nxt), _ptr(nbr), _ptr(grid),
+                           _ptr(dead), _ptr(alive), _ptr(dying), born, survive, C, _stream(stream))
+    if st:
+        ctx._check(st, "gen_step")
 
 
 def checksum_i32(vals, out, stream=None):

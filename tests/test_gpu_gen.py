@@ -18,17 +18,18 @@ def ctx():
     c.close()
 
 
+@pytest.mark.parametrize("fused", [True, False])
 @pytest.mark.parametrize("variant", VARIANTS)
 @pytest.mark.parametrize("W,H,gens,rule,torus", [(256, 256, 60, ("2", "345", 4), False),
                                                  (77, 45, 40, ("3", "23", 2), False),
                                                  (64, 64, 33, ("34", "34", 6), True)])
-def test_gen_parity(ctx, variant, W, H, gens, rule, torus):
+def test_gen_parity(ctx, variant, W, H, gens, rule, torus, fused):
     born, surv, C = rule
     s0 = synth.soup(W, H, seed=42)
     st_ref, ctr_ref, hist_ref, _ = oracle.gen_run(W, H, s0, gens, born, surv, C, torus)
     g = apps.Gen(ctx, W, H, s0, variant, born, surv, C, torus)
     for _ in range(gens):
-        g.gen()
+        g.gen(fused=fused)
     st = g.current.cpu().numpy()
     assert np.array_equal(st, st_ref)
     ctr, typ = g.counters()

@@ -19,15 +19,16 @@ def ctx():
     c.close()
 
 
+@pytest.mark.parametrize("fused", [True, False])
 @pytest.mark.parametrize("variant", VARIANTS)
 @pytest.mark.parametrize("W,H,gens,torus", [(256, 256, 100, False), (37, 23, 30, False), (64, 48, 25, True)])
-def test_gol_parity(ctx, variant, W, H, gens, torus):
+def test_gol_parity(ctx, variant, W, H, gens, torus, fused):
     g0 = synth.soup(W, H, seed=42)
     st_ref, ctr_ref, pop_ref, _ = oracle.gol_run(W, H, g0, gens, torus)
     g = apps.Gol(ctx, W, H, g0, variant, torus)
     pops = []
     for _ in range(gens):
-        g.gen()
+        g.gen(fused=fused)
         pops.append(int(g.current.sum().item()))
     assert np.array_equal(g.current.cpu().numpy(), st_ref)
     ctr, typ = g.counters()

@@ -90,9 +90,10 @@ def bench_gol(ctx, quick):
                 g.gen(stream=s)
         ms = ev_time(graph.replay, 5) / gens
         ms_eager = ev_time(g.gen, 50)
+        ms_unfused = ev_time(lambda: g.gen(fused=False), 50)
         # 8 B ptr + 1 B nbr + 1 B state out + 4 B counter r/w per next() call
         record("gol", "256x256, 100 gens (CUDA graph of 100 generations)", v, W * H, ms, 14, "GB/s", "l2/latency",
-               dict(ms_per_gen_eager=ms_eager), cpu)
+               dict(ms_per_gen_eager=ms_eager, ms_per_gen_eager_unfused=ms_unfused), cpu)
         del g, graph
     ctx.reset()
 
@@ -109,7 +110,12 @@ def bench_gen(ctx, quick):
         sv = s0 if Wv == W else synth.soup(Wv, Wv, seed=42)
         g = apps.Gen(ctx, Wv, Wv, sv, v)
         ms = ev_time(g.gen, gens)
-        record("gen", f"{Wv}x{Wv} B2/S345/C4", v, Wv * Wv, ms, 14, "GB/s", "hbm", None, cpu)
+        g2 = apps.Gen(ctx, Wv, Wv, sv, v)
+        ms_unfused = ev_time(lambda: g2.gen(fused=False), gens)
+        # fused step per cell: 8 B ptr + 16 B object r/w + ~1 B state read (9 neighbours from L1/L2) + 1 B write
+        record("gen", f"{Wv}x{Wv} B2/S345/C4 (fused step)", v, Wv * Wv, ms, 14, "GB/s", "hbm",
+               dict(ms_unfused=ms_unfused), cpu)
+        del g2
         del g
         ctx.reset()
 
