@@ -65,7 +65,10 @@ typedef enum {
   VF_ERR_UNSUPPORTED = 7      /* valid but not implemented for this app/variant        */
 } vf_status;
 
-typedef enum { VF_CUDA = 0, VF_SHAREDOA = 1, VF_COAL = 2, VF_TYPEPTR = 3 } vf_variant;
+/* VF_CONCORD is the paper's comparison point (§7): a type tag
+ * embedded in every object, read per call and switched on (apps with an
+ * embedded tag only: VF_APP_MICRO; others return VF_ERR_UNSUPPORTED). */
+typedef enum { VF_CUDA = 0, VF_SHAREDOA = 1, VF_COAL = 2, VF_TYPEPTR = 3, VF_CONCORD = 4 } vf_variant;
 
 /* Workload apps compiled into libvf.so (GPUs cannot load code at run time,
  * so every class whose virtual methods a kernel may call is compiled into
@@ -119,7 +122,8 @@ typedef struct {
  * update(): a = sum_{j != idx, ascending j} m_j d / (r^2+eps2[type])^{3/2}
  * with r2 = fmaf(dx,dx,fmaf(dy,dy,fmaf(dz,dz,eps2))), 1/(r2*sqrt(r2)),
  * a = fmaf(d, m_j*inv, a); Dust: v *= damp; v = fmaf(dt,a,v);
- * pout[idx] = (fmaf(dt,v,x), ..., m). Reads pin[0..N), writes pout[idx]. */
+ * pout[idx] = (fmaf(dt,v,x), ..., m). Reads pin[0..N), writes pout[idx].
+ * Precondition (IEEE-exact results): eps2[t] >= 1e-20 and |coordinates| < 1e11. */
 enum { VF_NBODY_UPDATE = 0, VF_NBODY_GET = 1 };
 typedef struct {
   const float4_t* pin_dev;  /* N float4, positions at the start of the step (all bodies) */
@@ -166,7 +170,9 @@ typedef struct {
   uint32_t id_base;
 } vf_traf_get_args;
 
-/* Methods of VF_APP_MICRO (args structs are passed by value, see dispatch). */
+/* Methods of VF_APP_MICRO (args structs are passed by value, see dispatch).
+ * Layout {vptr, i32 val, u32 tag}: tag = the class id, Concord's embedded
+ * type field (VF_CONCORD reads it; the other variants ignore it). */
 enum { VF_MICRO_APPLY = 0, /* args: none                                       */
        VF_MICRO_GET = 1 }; /* args: vf_micro_get_args — out_dev[i] = objs[i].val */
 typedef struct { int32_t* out_dev; } vf_micro_get_args;
@@ -369,6 +375,9 @@ vf_status vf_dispatch_coal(vf_ctx* ctx, uint32_t app, uint32_t method, const uin
 vf_status vf_dispatch_typeptr(vf_ctx* ctx, uint32_t app, uint32_t method,
                               const uint64_t* objs_dev, uint64_t n, const void* args,
                               size_t args_bytes, void* stream);
+/* Concord (embedded type tag + switch, one object per thread). */
+vf_status vf_dispatch_concord(vf_ctx* ctx, uint32_t app, uint32_t method, const uint64_t* objs_dev,
+                              uint64_t n, const void* args, size_t args_bytes, void* stream);
 /* Same, variant as a parameter. */
 vf_status vf_dispatch(vf_ctx* ctx, vf_variant v, uint32_t app, uint32_t method,
                       const uint64_t* objs_dev, uint64_t n, const void* args, size_t args_bytes,
@@ -428,6 +437,16 @@ vf_status vf_graph_bfs_init(uint64_t V, int32_t* depth_dev, uint32_t src, const 
 vf_status vf_iota_u32(uint64_t n, uint32_t* x_dev, void* stream);
 vf_status vf_fill_f32(uint64_t n, float* x_dev, float value, void* stream);
 
+/* BRANCH ceiling of the microbenchmark (§8.3: "decides which
+ * function to call based on register values and does not access memory for
+ * the function call"): no objects; for i in [0, n): t = the type config 2
+ * gives object i, computed in registers from (seed, order, T, k) with the
+ * synth recipe (order 0 random: t = floor(splitmix64(seed ^ 1<<56 ^ i) * T /
+ * 2^64); 1 sorted: floor(i*T/n); 2 k-per-warp: (i mod 32) mod k); then a
+ * switch on t adds t+1 to vals_dev[i] (int32). */
+vf_status vf_micro_branch(uint64_t n, uint32_t T, int order, uint64_t seed, uint32_t k, int32_t* vals_dev,
+                          void* stream);
+
 /* ---- utilities ---------------------------------------------------------- */
 /* sum over i of vals_dev[i] (int32, widened) into *out_dev (i64, device). */
 vf_status vf_checksum_i32(const int32_t* vals_dev, uint64_t n, long long* out_dev, void* stream);
@@ -438,7 +457,10 @@ vf_status vf_checksum_i32(const int32_t* vals_dev, uint64_t n, long long* out_de
  * each CTA tile by type in shared memory before the calls, 0 groups within
  * warps only; "pipeline" = 1 streams the pointer array through a TMA /
  * mbarrier ring in shared memory (regroup 0 only), 0 (default) uses plain
- * per-thread loads. VF_ERR_INVALID for unknown keys / values. */
+ * per-thread loads; "call" = 1 makes COAL / TYPEPTR CALL the resolved type's
+ * vFunc* indirectly (the paper's design, Table 1 row C, Fig. 5b line 4), 0
+ * (default) groups lanes by type and calls each body directly.
+ * VF_ERR_INVALID for unknown keys / values. */
 vf_status vf_set_tuning(const char* key, int value);
 /* Number of libvf kernel launches issued since load (for bench accounting). */
 uint64_t vf_launch_count(void);

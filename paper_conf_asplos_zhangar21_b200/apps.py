@@ -26,10 +26,15 @@ class Micro:
     val = init_i; after R steps val_i = init_i + R (t(i)+1).
     """
 
+    # variants beyond the four of vf.h: comparison points of the paper
+    #   concord       embedded type tag + switch (§7 P:1646-1653), typed arenas
+    #   typeptr_heap  TypePointer tags on device-heap `new` objects (§8.2 Fig. 11, P:2749-2757)
+    EXTRA = {"typeptr_heap": vf.TYPEPTR}
+
     def __init__(self, ctx: vf.Ctx, n: int, T: int, order: str = "random", seed: int = 42,
                  variant: str = "typeptr", k: int | None = None, types_np=None, init_np=None):
         self.ctx, self.n, self.T, self.variant = ctx, n, T, variant
-        self.v = vf.VARIANTS[variant]
+        self.v = self.EXTRA[variant] if variant in self.EXTRA else vf.VARIANTS[variant]
         dev = _dev(ctx.device)
         if types_np is None:
             types_np = synth.micro_types(n, T, order, seed=seed, k=k)
@@ -37,8 +42,8 @@ class Micro:
             init_np = synth.micro_init(n, seed=seed)
         self.types = torch.from_numpy(types_np.astype(np.int32)).to(dev)
         init = torch.from_numpy(init_np.astype(np.int32)).to(dev)
-        if variant == "cuda":
-            self.objs = ctx.alloc_cuda(vf.APP_MICRO, self.types, init)
+        if variant in ("cuda", "typeptr_heap"):
+            self.objs = ctx.alloc_cuda(vf.APP_MICRO, self.types, init, tag=(variant == "typeptr_heap"))
         else:
             self.objs = ctx.alloc_typed_batch(vf.APP_MICRO, self.types, init, tag=(variant == "typeptr"))
         torch.cuda.synchronize(dev)
@@ -56,6 +61,25 @@ class Micro:
         self.ctx.dispatch(self.v, vf.APP_MICRO, vf.MICRO_GET, self.objs,
                           vf.micro_get_args(out.data_ptr()), stream=stream)
         return out
+
+
+class MicroBranch:
+    """BRANCH ceiling of config 2 (§8.3): no objects, the type comes
+    from registers, a switch picks the addition (vf_micro_branch)."""
+
+    def __init__(self, ctx: vf.Ctx, n: int, T: int, order: str = "random", seed: int = 42, k: int | None = None,
+                 init_np=None):
+        self.n, self.T, self.order, self.seed = n, T, order, seed
+        self.k = (T if k is None else k) if order == "kperwarp" else 1
+        if init_np is None:
+            init_np = synth.micro_init(n, seed=seed)
+        self.vals = torch.from_numpy(init_np.astype(np.int32)).to(_dev(ctx.device))
+
+    def step(self, stream=None):
+        vf.micro_branch(self.vals, self.T, self.order, self.seed, self.k, stream)
+
+    def values(self, out=None, stream=None):
+        return self.vals
 
 
 class Gol:

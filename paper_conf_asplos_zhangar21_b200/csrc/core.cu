@@ -414,6 +414,9 @@ vf_status vf_set_tuning(const char* key, int value) {
   } else if (!strcmp(key, "pipeline")) {
     if (value < 0 || value > 1) return VF_ERR_INVALID;
     tuning().pipeline = value;
+  } else if (!strcmp(key, "call")) {
+    if (value < 0 || value > 1) return VF_ERR_INVALID;
+    tuning().call = value;
   } else {
     return VF_ERR_INVALID;
   }
@@ -668,7 +671,7 @@ vf_status vf_resolve(vf_ctx* c, uint32_t app, vf_variant v, const uint64_t* ptrs
                      uint32_t* types_out_dev, void* stream) {
   vf_status st = check_app(c, app);
   if (st) return st;
-  if ((unsigned)v > VF_TYPEPTR) return fail(c, VF_ERR_INVALID, "variant %d", (int)v);
+  if ((unsigned)v > VF_CONCORD) return fail(c, VF_ERR_INVALID, "variant %d", (int)v);
   if ((st = set_device(c)) || (st = ensure_vptrs(c, app))) return st;
   if (v == VF_COAL && c->tables[app].K > VF_MAX_RANGES)
     return fail(c, VF_ERR_TABLE_FULL, "K = %u > %u", c->tables[app].K, VF_MAX_RANGES);
@@ -680,7 +683,7 @@ vf_status vf_verify_types(vf_ctx* c, uint32_t app, vf_variant v, const uint64_t*
                           uint64_t n, unsigned long long* mism_dev, void* stream) {
   vf_status st = check_app(c, app);
   if (st) return st;
-  if ((unsigned)v > VF_TYPEPTR) return fail(c, VF_ERR_INVALID, "variant %d", (int)v);
+  if ((unsigned)v > VF_CONCORD) return fail(c, VF_ERR_INVALID, "variant %d", (int)v);
   if ((st = set_device(c)) || (st = ensure_vptrs(c, app))) return st;
   if (v == VF_COAL && c->tables[app].K > VF_MAX_RANGES)
     return fail(c, VF_ERR_TABLE_FULL, "K = %u > %u", c->tables[app].K, VF_MAX_RANGES);
@@ -694,7 +697,7 @@ vf_status vf_dispatch(vf_ctx* c, vf_variant v, uint32_t app, uint32_t method,
   vf_status st = check_app(c, app);
   if (st) return st;
   const AppOps* ops = app_ops(app);
-  if ((unsigned)v > VF_TYPEPTR) return fail(c, VF_ERR_INVALID, "variant %d", (int)v);
+  if ((unsigned)v > VF_CONCORD) return fail(c, VF_ERR_INVALID, "variant %d", (int)v);
   if (method >= ops->nmethods) return fail(c, VF_ERR_INVALID, "method %u of app %s", method, ops->name);
   if (args_bytes > VF_MAX_ARGS_BYTES || (args_bytes && !args))
     return fail(c, VF_ERR_INVALID, "args_bytes %zu", args_bytes);
@@ -707,8 +710,16 @@ vf_status vf_dispatch(vf_ctx* c, vf_variant v, uint32_t app, uint32_t method,
   ArgBlob blob;
   memset(&blob, 0, sizeof blob);
   if (args_bytes) memcpy(blob.b, args, args_bytes);
-  CUDA_TRY(c, ops->dispatch((int)v, method, objs_dev, n, blob, dev_table(c, app), S(stream)));
+  const cudaError_t e = ops->dispatch((int)v, method, objs_dev, n, blob, dev_table(c, app), S(stream));
+  if (e == cudaErrorNotSupported)
+    return fail(c, VF_ERR_UNSUPPORTED, "app %s has no embedded type tag (Concord)", ops->name);
+  CUDA_TRY(c, e);
   return VF_OK;
+}
+
+vf_status vf_dispatch_concord(vf_ctx* c, uint32_t app, uint32_t m, const uint64_t* o, uint64_t n, const void* a,
+                              size_t ab, void* s) {
+  return vf_dispatch(c, VF_CONCORD, app, m, o, n, a, ab, s);
 }
 
 vf_status vf_ray_render(vf_ctx* c, vf_variant v, const uint64_t* shapes_dev, uint32_t S, uint32_t W,

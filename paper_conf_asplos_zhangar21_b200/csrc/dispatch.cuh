@@ -21,6 +21,7 @@
 #include <stdint.h>
 
 #include <new>
+#include <type_traits>
 
 #include "vf_internal.h"
 
@@ -533,6 +534,101 @@ __global__ void __launch_bounds__(kBlock) k_dispatch_sorted(const uint64_t* __re
   }
 }
 
+// ---------------------------------------------------------------------------
+// Comparison points of the paper (§7, §8.3, Table 1
+// row C): Concord's embedded type tag + switch, and the paper-faithful
+// COAL / TypePointer that still CALL the looked-up vFunc* indirectly.
+// ---------------------------------------------------------------------------
+
+// Apps with an embedded type tag (Concord) define kTagOffset (byte offset of a
+// u32 type id inside every object); others get -1 (VF_ERR_UNSUPPORTED).
+template <class A, class = void>
+struct TagOffset {
+  static constexpr int value = -1;
+};
+template <class A>
+struct TagOffset<A, std::void_t<decltype(A::kTagOffset)>> {
+  static constexpr int value = A::kTagOffset;
+};
+
+// Concord [6]: "a type field is embedded in each object ... the
+// compiler inserts a switch statement, which reads the embedded type tag, then
+// jumps to the appropriate function body". One object per thread, a plain
+// C++ switch (compiled to a jump table / compare tree), no warp grouping.
+#define VF_CASE(k)                                                                     \
+  case k:                                                                              \
+    if constexpr (k < App::kTypes)                                                     \
+      App::template dcall<M, k>(reinterpret_cast<typename App::template Type<k>*>(a), i, args); \
+    break;
+template <class App, int M>
+__device__ __forceinline__ void concord_switch(uint32_t t, uint64_t a, uint64_t i, const ArgBlob& args) {
+  static_assert(App::kTypes <= 32, "switch covers 32 cases");
+  switch (t) {
+    VF_CASE(0) VF_CASE(1) VF_CASE(2) VF_CASE(3) VF_CASE(4) VF_CASE(5) VF_CASE(6) VF_CASE(7)
+    VF_CASE(8) VF_CASE(9) VF_CASE(10) VF_CASE(11) VF_CASE(12) VF_CASE(13) VF_CASE(14) VF_CASE(15)
+    VF_CASE(16) VF_CASE(17) VF_CASE(18) VF_CASE(19) VF_CASE(20) VF_CASE(21) VF_CASE(22) VF_CASE(23)
+    VF_CASE(24) VF_CASE(25) VF_CASE(26) VF_CASE(27) VF_CASE(28) VF_CASE(29) VF_CASE(30) VF_CASE(31)
+    default: break;
+  }
+}
+#undef VF_CASE
+
+template <class App, int M>
+__global__ void __launch_bounds__(kBlock) k_dispatch_concord(const uint64_t* __restrict__ objs, uint64_t n,
+                                                              ArgBlob args) {
+  const uint64_t i = (uint64_t)blockIdx.x * kBlock + threadIdx.x;
+  if (i >= n) return;
+  const uint64_t p = ldg_u64(objs + i);
+  if (!p) return;
+  const uint64_t a = strip(p);
+  const uint32_t t = *reinterpret_cast<const uint32_t*>(a + TagOffset<App>::value);  // the embedded tag
+  concord_switch<App, M>(t, a, i, args);
+}
+
+// Paper-faithful COAL / TypePointer (vf_set_tuning("call", 1)): after the type
+// is resolved from the pointer, the vFunc* is fetched from a per-CTA function
+// table (Fig. 5b lines 2-3, staged in shared memory) and CALLed indirectly
+// (line 4: "CALL R5"), one object per thread, no grouping.
+template <class App, int M, int K>
+__device__ __noinline__ void thunk(uint64_t a, uint64_t i, const ArgBlob* args) {
+  App::template dcall<M, K>(reinterpret_cast<typename App::template Type<K>*>(a), i, *args);
+}
+using ThunkFn = void (*)(uint64_t, uint64_t, const ArgBlob*);
+template <class App, int M, int K = 0>
+__device__ __forceinline__ void fill_thunks(ThunkFn* tab) {
+  if constexpr (K < App::kTypes) {
+    tab[K] = &thunk<App, M, K>;
+    fill_thunks<App, M, K + 1>(tab);
+  }
+}
+
+template <class App, int M, class R>
+__global__ void __launch_bounds__(kBlock) k_dispatch_indirect(const uint64_t* __restrict__ objs, uint64_t n,
+                                                               ArgBlob args, DevTable tbl) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  __shared__ ThunkFn s_fn[App::kTypes];
+  __shared__ ArgBlob s_args;
+  if constexpr (R::kNeedsTable) R::stage(smem, tbl);
+  if (threadIdx.x == 0) {
+    fill_thunks<App, M>(s_fn);
+    s_args = args;
+  }
+  __syncthreads();
+  uint32_t hint = 0;
+  for (uint64_t i = (uint64_t)blockIdx.x * kBlock + threadIdx.x; i < n; i += (uint64_t)gridDim.x * kBlock) {
+    const uint64_t p = ldg_u64(objs + i);
+    if (!p) continue;
+    uint64_t a;
+    const uint32_t t = R::resolve(smem, tbl.P, p, a, hint);
+    if (t < (uint32_t)App::kTypes) {
+      const ThunkFn f = s_fn[t];  // vFunc* = table[type]
+      f(a, i, &s_args);           // indirect CALL
+    } else {
+      App::template vcall<M>(reinterpret_cast<typename App::Base*>(a), i, args);  // fallback
+    }
+  }
+}
+
 // CUDA / SharedOA dispatch: the plain C++ virtual call, one object per thread,
 // as the user writes it (`objs[i]->f()`).
 template <class App, int M>
@@ -595,6 +691,13 @@ __device__ __forceinline__ uint32_t resolve_rule(int variant, const unsigned cha
   uint32_t hint = 0;
   if (variant == VF_TYPEPTR) return ResolveTP::resolve(smem, tbl.P, p, a, hint);
   if (variant == VF_COAL) return ResolveCOAL::resolve(smem, tbl.P, p, a, hint);
+  if (variant == VF_CONCORD) {
+    if constexpr (TagOffset<App>::value >= 0) {
+      const uint32_t t = *reinterpret_cast<const uint32_t*>(strip(p) + TagOffset<App>::value);
+      return t < tbl.ntypes ? t : kNF;
+    }
+    return kNF;
+  }
   // CUDA / SharedOA: the embedded vTable* (Fig. 1a load A), mapped to a type id
   const uint64_t vp = *reinterpret_cast<const uint64_t*>(p);
   for (uint32_t k = 0; k < tbl.ntypes; ++k)
@@ -763,18 +866,47 @@ cudaError_t launch_grouped_tuned(const uint64_t* objs, uint64_t n, const ArgBlob
   return launch_grouped_pf<App, M, R, 1>(pf, objs, n, args, tbl, s);
 }
 
+template <class App, int M, class R>
+cudaError_t launch_indirect(const uint64_t* objs, uint64_t n, const ArgBlob& args, const DevTable& tbl,
+                            cudaStream_t s) {
+  auto kern = k_dispatch_indirect<App, M, R>;
+  const size_t sm = R::kNeedsTable ? table_smem(tbl) : 0;
+  static int occ = -1;
+  static size_t occ_sm = ~(size_t)0;
+  if (occ < 0 || occ_sm != sm) {
+    if (sm > 40 * 1024) cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kBlock, sm);
+    if (occ < 1) occ = 1;
+    occ_sm = sm;
+  }
+  kern<<<grid_for(n, kBlock, (uint64_t)num_sms() * occ), kBlock, sm, s>>>(objs, n, args, tbl);
+  note_launch();
+  return cudaGetLastError();
+}
+
 template <class App, int M>
 cudaError_t dispatch_method(int variant, const uint64_t* objs, uint64_t n, const ArgBlob& args,
                             const DevTable& tbl, cudaStream_t s) {
   if (n == 0) return cudaSuccess;
+  const bool indirect = tuning().call != 0;
   switch (variant) {
     case VF_CUDA:
     case VF_SHAREDOA:
       return launch_virtual<App, M>(objs, n, args, s);
     case VF_COAL:
+      if (indirect) return launch_indirect<App, M, ResolveCOAL>(objs, n, args, tbl, s);
       return launch_grouped_tuned<App, M, ResolveCOAL>(objs, n, args, tbl, s);
     case VF_TYPEPTR:
+      if (indirect) return launch_indirect<App, M, ResolveTP>(objs, n, args, tbl, s);
       return launch_grouped_tuned<App, M, ResolveTP>(objs, n, args, tbl, s);
+    case VF_CONCORD:
+      if constexpr (TagOffset<App>::value >= 0) {
+        k_dispatch_concord<App, M><<<grid_for(n, kBlock, ~0u), kBlock, 0, s>>>(objs, n, args);
+        note_launch();
+        return cudaGetLastError();
+      } else {
+        return cudaErrorNotSupported;
+      }
   }
   return cudaErrorInvalidValue;
 }

@@ -85,6 +85,7 @@ struct Tuning {
   int prefetch = -1;  // 0 none, 1 prefetch.global.L1, 2 L1-allocating warm load
   int pipeline = 0;   // 1: TMA-pipelined pointer stream (k_dispatch_pipe), 0: plain loads
   int regroup = 1;    // 1: CTA-level counting sort of each tile by type (k_dispatch_sorted)
+  int call = 0;       // COAL / TypePointer: 0 grouped direct call, 1 indirect CALL via vFunc* table
 };
 Tuning& tuning();
 

@@ -17,8 +17,9 @@ SO = os.path.join(PKG, "libvf.so")
 
 # enums mirrored from include/vf.h
 VF_OK = 0
-CUDA, SHAREDOA, COAL, TYPEPTR = 0, 1, 2, 3
-VARIANTS = {"cuda": CUDA, "sharedoa": SHAREDOA, "coal": COAL, "typeptr": TYPEPTR}
+CUDA, SHAREDOA, COAL, TYPEPTR, CONCORD = 0, 1, 2, 3, 4
+VARIANTS = {"cuda": CUDA, "sharedoa": SHAREDOA, "coal": COAL, "typeptr": TYPEPTR, "concord": CONCORD}
+ORDERS = {"random": 0, "sorted": 1, "kperwarp": 2}
 APP_MICRO, APP_GOL, APP_GEN, APP_GRAPH = 0, 1, 2, 3
 MICRO_APPLY, MICRO_GET = 0, 1
 GOL_NEXT, GOL_GET = 0, 1
@@ -39,6 +40,7 @@ SYMBOLS = [
     "vf_dispatch_sharedoa", "vf_dispatch_coal", "vf_dispatch_typeptr", "vf_dispatch",
     "vf_gol_neighbors", "vf_gol_swap", "vf_gen_swap", "vf_checksum_i32", "vf_launch_count", "vf_set_tuning",
     "vf_graph_bfs_init", "vf_iota_u32", "vf_fill_f32", "vf_ray_render", "vf_gol_step", "vf_gen_step",
+    "vf_dispatch_concord", "vf_micro_branch",
 ]
 APP_RAY = 4
 APP_TRAF = 5
@@ -200,6 +202,8 @@ def lib(required: bool = True):
         "vf_fill_f32": (I, [U64, P, ctypes.c_float, P]),
         "vf_ray_render": (I, [P, I, P, U32, U32, U32, U32, U32, P, P, P, P, P]),
         "vf_gol_step": (I, [P, I, U32, U32, I, P, P, P, P, P, P, P]),
+        "vf_dispatch_concord": (I, [P, U32, U32, P, U64, P, ctypes.c_size_t, P]),
+        "vf_micro_branch": (I, [U64, U32, I, U64, U32, P, P]),
         "vf_gen_step": (I, [P, I, U32, U32, I, P, P, P, P, P, P, P, U32, U32, U32, P]),
     }
     for name, (res, args) in sig.items():
@@ -406,6 +410,13 @@ def gen_step(ctx: Ctx, variant: int, W, H, torus, prev, nxt, nbr, grid, dead, al
                            _ptr(dead), _ptr(alive), _ptr(dying), born, survive, C, _stream(stream))
     if st:
         ctx._check(st, "gen_step")
+
+
+def micro_branch(vals, T: int, order: str, seed: int, k: int = 1, stream=None):
+    """BRANCH ceiling (vf.h vf_micro_branch): vals[i] += t(i)+1, t from registers."""
+    st = lib().vf_micro_branch(vals.numel(), T, ORDERS[order], seed, k, _ptr(vals), _stream(stream))
+    if st:
+        raise VFError(st, "micro_branch")
 
 
 def checksum_i32(vals, out, stream=None):

@@ -200,3 +200,56 @@ def test_micro_full_size_sampled():
 
 def ctx_verify(c, m):
     return c.verify(vf.APP_MICRO, m.v, m.objs)
+
+
+# ---- the paper's comparison points (§7, §8.2 Fig. 11, §8.3 Fig. 12, Table 1 row C)
+@pytest.mark.parametrize("variant", ["concord", "typeptr_heap"])
+@pytest.mark.parametrize("T,order", [(1, "random"), (4, "random"), (4, "sorted"), (32, "random"), (5, "kperwarp")])
+def test_micro_comparison_variants(ctx, variant, T, order):
+    n, R = 4096 * 5 + 77, 3
+    types = synth.micro_types(n, T, order, seed=3, k=min(T, 5))
+    init = synth.micro_init(n, seed=3)
+    ref, _ = oracle.micro_run(types, init, T, R)
+    m = apps.Micro(ctx, n, T, variant=variant, types_np=types, init_np=init)
+    for _ in range(R):
+        m.step()
+    assert np.array_equal(m.values().cpu().numpy(), ref)
+    assert ctx.verify(vf.APP_MICRO, m.v, m.objs) == 0  # concord: the embedded tag names the right class
+
+
+@pytest.mark.parametrize("variant", ["coal", "typeptr"])
+@pytest.mark.parametrize("T,order", [(4, "random"), (32, "random"), (3, "sorted")])
+def test_micro_indirect_call_flavour(ctx, variant, T, order):
+    """vf_set_tuning("call", 1): resolved type -> vFunc* table -> indirect CALL (the paper's design)."""
+    n, R = 4096 * 7 + 5, 2
+    types = synth.micro_types(n, T, order, seed=8)
+    init = synth.micro_init(n, seed=8)
+    ref, _ = oracle.micro_run(types, init, T, R)
+    vf.set_tuning("call", 1)
+    try:
+        m = apps.Micro(ctx, n, T, variant=variant, types_np=types, init_np=init)
+        for _ in range(R):
+            m.step()
+        assert np.array_equal(m.values().cpu().numpy(), ref)
+    finally:
+        vf.set_tuning("call", 0)
+
+
+@pytest.mark.parametrize("T,order,k", [(1, "random", 1), (4, "random", 1), (32, "random", 1), (4, "sorted", 1),
+                                       (32, "kperwarp", 7)])
+def test_micro_branch_ceiling_closed_form(ctx, T, order, k):
+    """BRANCH computes the same types in registers: val_i = init_i + R(t_i+1)."""
+    n, R = 100_003, 4
+    types = synth.micro_types(n, T, order, seed=11, k=k)
+    init = synth.micro_init(n, seed=11)
+    b = apps.MicroBranch(ctx, n, T, order, seed=11, k=k, init_np=init)
+    for _ in range(R):
+        b.step()
+    assert np.array_equal(b.values().cpu().numpy(), init.astype(np.int64) + R * (types.astype(np.int64) + 1))
+
+
+def test_concord_unsupported_without_tag(ctx):
+    g = apps.Gol(ctx, 8, 8, synth.soup(8, 8, seed=1), "sharedoa")
+    with pytest.raises(vf.VFError) as e:
+        ctx.dispatch(vf.CONCORD, vf.APP_GOL, vf.GOL_NEXT, g.grid, g.args[0])
+    assert e.value.status == 7

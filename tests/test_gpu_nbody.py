@@ -74,3 +74,26 @@ def test_nbody_block_shards_reassemble(ctx):
     assert np.array_equal(ranks[0].positions(), p_ref)
     v = np.concatenate([nb.velocities() for nb in ranks])
     assert np.array_equal(v, v_ref)
+
+
+@pytest.mark.parametrize("variant", ["cuda", "typeptr"])
+def test_nbody_fast_math_range_edges(ctx, variant):
+    """The branch-free IEEE sqrt / reciprocal (app_nbody.cu) at the edges of the
+    documented range: eps2 = 1e-20 with coincident bodies, separations up to
+    1e10, tiny masses (finite, NaN-free accelerations) -> still bit-exact vs the oracle."""
+    N = 512
+    s = synth.nbody_system(N, seed=77)
+    s["eps2"][:] = np.array([1e-20, 1e-12, 0.5], np.float32)
+    rng = np.random.default_rng(5)
+    s["pos"][:64, :3] = 0.0  # coincident cluster: r2 == eps2 exactly
+    s["pos"][64:128, :3] = rng.uniform(-1e10, 1e10, (64, 3)).astype(np.float32)
+    s["pos"][128:192, :3] = rng.uniform(-1e-8, 1e-8, (64, 3)).astype(np.float32)
+    s["pos"][:, 3] = (10.0 ** rng.uniform(-15, -10, N)).astype(np.float32)
+    p_ref, v_ref, _ = oracle.nbody_run(s, 2)
+    nb = Nbody(ctx, s, variant)
+    for _ in range(2):
+        nb.step()
+    p, v = nb.positions(), nb.velocities()
+    assert np.isfinite(p_ref).all() and np.isfinite(v_ref).all()
+    assert np.array_equal(p.view(np.uint32), p_ref.view(np.uint32))
+    assert np.array_equal(v.view(np.uint32), v_ref.view(np.uint32))
