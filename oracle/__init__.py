@@ -27,7 +27,7 @@ import numpy as np
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 SO = os.path.join(HERE, "liboracle.so")
-SOURCES = ["alloc.cpp", "micro.cpp", "gol.cpp", "gen.cpp", "graph.cpp", "ray.cpp", "traf.cpp", "nbody.cpp", "stut.cpp"]
+SOURCES = ["alloc.cpp", "micro.cpp", "gol.cpp", "gen.cpp", "graph.cpp", "ray.cpp", "traf.cpp", "nbody.cpp", "stut.cpp", "collide.cpp"]
 NOT_FOUND = 0xFFFFFFFF
 
 
@@ -102,6 +102,9 @@ def lib():
         F = ctypes.c_float
         L.oracle_stut_run.argtypes = [U32, P, P, P, P, U32, P, P, P, P, P, P, U32, F, F, F, F, ctypes.c_int, P, P, P,
                                       ctypes.POINTER(ctypes.c_double)]
+        L.oracle_collide_run.restype = ctypes.c_int
+        L.oracle_collide_run.argtypes = [U32, P, P, P, U32, U32, F, F, F, P, F, ctypes.c_int, P, P, P,
+                                         ctypes.POINTER(ctypes.c_double)]
         L.oracle_max_threads.restype = ctypes.c_int
         _lib = L
     return _lib
@@ -335,3 +338,23 @@ def stut_run(w: dict, steps: int, threads: int = 1):
     if rc:
         raise ValueError(f"oracle_stut_run rc={rc}")
     return po, vo, bo[:S], secs.value
+
+
+def collide_run(sys_: dict, steps: int, threads: int = 1):
+    """sys_ = synth.collide_system(...); returns (pos float32[N,4], vel float32[N,4], calls, seconds)."""
+    types = np.ascontiguousarray(sys_["types"], np.uint32)
+    pos = np.ascontiguousarray(sys_["pos"], np.float32)
+    vel = np.ascontiguousarray(sys_["vel"], np.float32)
+    eps2 = np.ascontiguousarray(sys_["eps2"], np.float32)
+    N = len(types)
+    po = np.zeros((N, 4), np.float32)
+    vo = np.zeros((N, 4), np.float32)
+    calls = ctypes.c_uint64()
+    sec = ctypes.c_double()
+    rc = lib().oracle_collide_run(N, types.ctypes.data, pos.ctypes.data, vel.ctypes.data, steps, int(sys_["G"]),
+                                  float(sys_["rc"]), float(sys_["rm"]), float(sys_["dt"]), eps2.ctypes.data,
+                                  float(sys_["damp"]), threads, po.ctypes.data, vo.ctypes.data, ctypes.byref(calls),
+                                  ctypes.byref(sec))
+    if rc:
+        raise ValueError(f"oracle_collide_run rc={rc}")
+    return po, vo, calls.value, sec.value

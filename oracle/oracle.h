@@ -171,6 +171,17 @@ int oracle_stut_run(uint32_t n, const uint32_t* types, const float* pos2, const 
                     uint32_t steps, float dt, float c, float v_pull, float brk, int threads,
                     float* pos_out, float* vel_out, uint8_t* broken_out, double* seconds);
 
+/* ---- Config 5 collision (readings G18/G19; see collide.cpp) --------------
+ * N bodies (types 0 Star, 1 Planet, 2 Dust; pos4 = x,y,z,m with m = 0 meaning
+ * inactive; vel4 = vx,vy,vz,unused) on a G^3 grid of cells of side rc:
+ * per step one virtual update() (cutoff rc softened gravity, nearest body
+ * within rm) and one virtual merge() (mutual nearest pairs: the smaller id
+ * absorbs the larger) per active body. calls_out = virtual calls issued. */
+int oracle_collide_run(uint32_t N, const uint32_t* types, const float* pos4, const float* vel4,
+                       uint32_t steps, uint32_t G, float rc, float rm, float dt, const float* eps2,
+                       float damp, int threads, float* pos_out, float* vel_out, uint64_t* calls_out,
+                       double* seconds);
+
 /* number of OpenMP threads actually available */
 int oracle_max_threads(void);
 

@@ -35,6 +35,7 @@ S_TRAF = 8      # traffic: vehicle placement / types
 S_TRAF_RNG = 9  # traffic: per-step slowdown draws (counter index = id<<24 ^ t)
 S_BODY = 10     # n-body initial conditions
 S_STUT = 11     # structure perturbation
+S_COLL = 12     # collision bodies
 
 
 def splitmix64(x: np.ndarray | int) -> np.ndarray:
@@ -387,3 +388,32 @@ def stut_custom(types, pos, mass, a, b, L0, k, vel=None, dt=0.01, damping=0.0, v
                 mass=np.asarray(mass, np.float32), a=a, b=b, L0=np.asarray(L0, np.float32),
                 k=np.asarray(k, np.float32), inc_offs=inc_offs, inc=inc, dt=np.float32(dt),
                 damping=np.float32(damping), v_pull=np.float32(v_pull), break_ratio=np.float32(break_ratio))
+
+
+
+# --------------------------------------------------------------------------
+# Config 5 collision (readings G18 / G19)
+# --------------------------------------------------------------------------
+COLL_EPS2 = np.array([0.02, 0.01, 0.005], np.float32)  # per type, in units of rc^2 = 1
+
+
+def collide_system(N: int, seed: int = 13, per_cell: float = 4.0, rm: float = 0.05, dt: float = 0.01,
+                   damp: float = 0.999, vmax: float = 0.5):
+    """N bodies uniform in [0, G)^3 with cells of side rc = 1 (G = ceil((N/per_cell)^(1/3))),
+    velocities uniform in [-vmax, vmax]^3, type uniform(3) (Star / Planet / Dust), masses as
+    the N-body system's; merge radius rm. vel is N x 4 (w unused)."""
+    G = max(1, int(np.ceil((N / per_cell) ** (1.0 / 3.0))))
+    i = np.arange(N, dtype=np.uint64)
+    r = [_unit(seed, S_COLL, i * np.uint64(8) + np.uint64(k)) for k in range(7)]
+    types = uniform(draw(seed, S_COLL, i + np.uint64(1 << 40)), 3)
+    pos = np.zeros((N, 4), np.float32)
+    for k in range(3):
+        pos[:, k] = np.float32(G) * r[k]
+    lo = np.array([m[0] for m in NBODY_MASS], np.float32)[types]
+    hi = np.array([m[1] for m in NBODY_MASS], np.float32)[types]
+    pos[:, 3] = lo + r[3] * (hi - lo)
+    vel = np.zeros((N, 4), np.float32)
+    for k in range(3):
+        vel[:, k] = np.float32(vmax) * (np.float32(2.0) * r[4 + k] - np.float32(1.0))
+    return dict(types=types, pos=pos, vel=vel, eps2=COLL_EPS2.copy(), dt=np.float32(dt), damp=np.float32(damp),
+                G=G, rc=np.float32(1.0), rm=np.float32(rm))
