@@ -346,13 +346,16 @@ def run_ours(args, rank, world, local):
 
     pk = peaks()
     hbm = pk.get("hbm_gbs")
+    peak_src = "MEASURED_PEAKS.json hbm_gbs (copy, burst), of measured"
+    if not hbm:  # file absent on this box: the profiling guide's stated fallback
+        hbm, peak_src = 6650.0, "B200_PROFILING.md fallback 6.65 TB/s (MEASURED_PEAKS.json absent), of fallback"
     kern = f"k_dispatch_grouped<micro,apply,{'ResolveTP' if args.variant == 'typeptr' else 'ResolveCOAL'}>" \
         if args.variant in ("coal", "typeptr") else "k_dispatch_virtual<micro,apply>"
     achieved = ALG_BYTES_PER_CALL * n / (step_ms / 1e3) / 1e9
     tr = ncu_traffic(f"micro_{args.variant}_T{args.T}_{args.order}")
     roof = {"bound": "hbm", "kernel": kern, "achieved": achieved, "peak": hbm, "unit": "GB/s",
             "frac": (achieved / hbm) if hbm else None,
-            "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy, burst)" if hbm else None,
+            "peak_source": peak_src,
             "traffic": tr,
             "alg_bytes_per_call": ALG_BYTES_PER_CALL,
             "layout_floor_bytes_per_call": LAYOUT_BYTES_PER_CALL,

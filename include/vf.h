@@ -82,7 +82,8 @@ enum {
   VF_APP_TRAF = 5,  /* config 5: Agent / PlainCell / LightCell / Car / Truck / Bus        */
   VF_APP_NBODY = 6, /* config 5: Body / Star / Planet / Dust (all-pairs N-body, G18)      */
   VF_APP_STUT = 7,  /* config 5: Element / Node / AnchorNode / AnchorPullNode / Spring   */
-  VF_APP_COUNT = 8
+  VF_APP_COLLIDE = 8, /* config 5: Body / Star / Planet / Dust (cutoff grid + merging, G19) */
+  VF_APP_COUNT = 9
 };
 
 /* Methods of VF_APP_STUT (Table 2 "structure" P:1524-1528, reading G17). Type
@@ -137,6 +138,51 @@ typedef struct {
   float* vel_out_dev;       /* 3 floats per body at (idx - idx_base)                     */
   uint32_t idx_base;
 } vf_nbody_get_args;
+
+/* Methods of VF_APP_COLLIDE (config 5 "collision" at 16M bodies; DynaSOAr's
+ * collision app [46], readings G18 / G19 in DESIGN.md). Type ids 0 Star,
+ * 1 Planet, 2 Dust; constructor argument {u32 idx, f32 vx, vy, vz} (the body
+ * keeps its velocity; positions+masses are float4 (x, y, z, m) arrays indexed
+ * by idx, m <= 0 = absorbed / inactive). One step, from the state P at its
+ * start: vf_collide_grid (non-virtual: uniform grid of cells of side rc, ids
+ * ascending per cell), then one virtual update() and one virtual merge() per
+ * active body:
+ *   update(): over the 27 neighbour cells in (z, y, x) order, bodies j != idx
+ *     in ascending id: d = p_j - p_i, d2 = fmaf(dx,dx,fmaf(dy,dy,dz*dz)); if
+ *     d2 < rc2: r2 = fmaf(dx,dx,fmaf(dy,dy,fmaf(dz,dz,eps2[type]))),
+ *     a = fmaf(d, m_j * (1/(r2*sqrt(r2))), a); the nearest j with d2 < rm2
+ *     (ties: smaller id) is near[idx] (-1 if none). Dust: v *= damp;
+ *     v = fmaf(dt,a,v); Pm[idx] = (fmaf(dt,v,x), m); Vm[idx] = v if near >= 0.
+ *   merge(): j = near[idx]; if near[j] == idx the smaller id absorbs:
+ *     m = m_i + m_j, x = fmaf(m_i,x_i,m_j*x_j)/m, v likewise (post-update
+ *     values); the larger id gets mass 0, velocity 0, position kept.
+ *     P[idx] = the result (Pm[idx] when there is no mutual partner).
+ * Same arithmetic as VF_APP_NBODY (IEEE-exact, no contraction). Preconditions:
+ * eps2[t] >= 1e-20, rc2 + eps2 <= 1e24, |coordinates| < 1e11. */
+enum { VF_COLLIDE_UPDATE = 0, VF_COLLIDE_MERGE = 1, VF_COLLIDE_GET = 2 };
+typedef struct {
+  const float4_t* P_dev;           /* N, start of step, by id (all bodies)            */
+  const float4_t* Ps_dev;          /* N, cell-sorted copy: Ps[e] = P[list[e]]          */
+  const uint32_t* list_dev;        /* ids in cell order, ascending within a cell       */
+  const uint32_t* cell_start_dev;  /* G^3 + 1 offsets into list                         */
+  float4_t* Pm_dev;                /* N, post-update position + mass, by id             */
+  float4_t* Vm_dev;                /* N, post-update velocity (written when near >= 0)  */
+  int32_t* near_dev;               /* N, nearest body within rm or -1                   */
+  uint32_t G;
+  float rc, rc2, rm2, dt;          /* rc2 = rc*rc, rm2 = rm*rm (fp32, host-rounded)     */
+  float eps2[3];
+  float damp;
+} vf_collide_update_args;
+typedef struct {
+  const float4_t* Pm_dev;
+  const float4_t* Vm_dev;
+  const int32_t* near_dev;
+  float4_t* P_dev;                 /* N, end of step, by id: this call writes P[idx]    */
+} vf_collide_merge_args;
+typedef struct {
+  float* vel_out_dev;              /* 3 floats per body at (idx - idx_base)              */
+  uint32_t idx_base;
+} vf_collide_get_args;
 
 /* Methods of VF_APP_TRAF (Table 2, reading G16). Type ids: 0
  * PlainCell, 1 LightCell (ctor arg {u32 cell, u32 phase}); 2 Car, 3 Truck,
@@ -427,6 +473,36 @@ vf_status vf_gen_step(vf_ctx* ctx, vf_variant v, uint32_t W, uint32_t H, int tor
 vf_status vf_ray_render(vf_ctx* ctx, vf_variant v, const uint64_t* shapes_dev, uint32_t S, uint32_t W,
                         uint32_t H, uint32_t row0, uint32_t nrows, const float* cam, const float* albedo,
                         float* rgb_dev, int32_t* hit_dev, void* stream);
+
+/* Collision step (0), non-virtual: the uniform grid and the dispatch order.
+ * For every body i with P[i].w > 0: cell (clamp(floor(x/rc)), clamp(floor(y/rc)),
+ * clamp(floor(z/rc))) of a G^3 grid, c = (z*G + y)*G + x; cell_start = the
+ * exclusive prefix sum of the cell counts; list[cell_start[c] ..) = the ids of
+ * cell c ascending; Ps[e] = P[list[e]]. Then order[k] = the objects of the
+ * owned ids [id_lo, id_hi) that are active, in cell order (spatially
+ * neighbouring bodies share a warp), null-padded to id_hi - id_lo entries
+ * (null pointers are skipped by every dispatch variant). *active_dev (if not
+ * NULL) += the number of owned active bodies (call accounting).
+ * Buffers are device memory owned by the caller; cell_count_dev must be all
+ * zero on entry and is left all zero; tmp_dev holds vf_collide_tmp_words(N, G)
+ * u32. 1 <= G <= 1024; VF_ERR_INVALID otherwise. */
+typedef struct {
+  uint32_t N, G;
+  float rc;
+  const float4_t* P_dev;          /* N                                          */
+  uint32_t* cell_of_dev;          /* N (0xFFFFFFFF = inactive)                  */
+  uint32_t* cell_count_dev;       /* G^3, zero on entry and on return           */
+  uint32_t* cell_start_dev;       /* G^3 + 1                                    */
+  uint32_t* list_dev;             /* N                                          */
+  float4_t* Ps_dev;               /* N                                          */
+  uint32_t* tmp_dev;              /* vf_collide_tmp_words(N, G)                 */
+  const uint64_t* objs_dev;       /* id_hi - id_lo: object of body id_lo + k     */
+  uint32_t id_lo, id_hi;
+  uint64_t* order_dev;            /* id_hi - id_lo                              */
+  unsigned long long* active_dev; /* may be NULL                                */
+} vf_collide_grid_args;
+uint64_t vf_collide_tmp_words(uint32_t N, uint32_t G);
+vf_status vf_collide_grid(const vf_collide_grid_args* args, void* stream);
 
 /* Graph helpers: BFS start state (depth = -1 except depth[src] = 0, queue =
  * src's nch work entries (vobj[src], chunks 0..nch-1), *count = nch), iota

@@ -32,7 +32,8 @@ def _headers():
 # contraction (every FMA is an explicit fmaf in the source), IEEE div/sqrt.
 PER_FILE = {"app_ray.cu": ["-fmad=false", "-prec-div=true", "-prec-sqrt=true", "-ftz=false"],
             "app_nbody.cu": ["-fmad=false", "-prec-div=true", "-prec-sqrt=true", "-ftz=false"],
-            "app_stut.cu": ["-fmad=false", "-prec-div=true", "-prec-sqrt=true", "-ftz=false"]}
+            "app_stut.cu": ["-fmad=false", "-prec-div=true", "-prec-sqrt=true", "-ftz=false"],
+            "app_collide.cu": ["-fmad=false", "-prec-div=true", "-prec-sqrt=true", "-ftz=false"]}
 
 
 def _compile(src: str, obj: str, verbose: bool) -> str:

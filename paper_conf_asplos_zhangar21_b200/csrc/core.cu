@@ -41,6 +41,7 @@ static const AppOps* app_ops(uint32_t app) {
     case VF_APP_TRAF: return app_traf();
     case VF_APP_NBODY: return app_nbody();
     case VF_APP_STUT: return app_stut();
+    case VF_APP_COLLIDE: return app_collide();
   }
   return nullptr;
 }

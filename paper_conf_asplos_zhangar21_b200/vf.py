@@ -40,7 +40,7 @@ SYMBOLS = [
     "vf_dispatch_sharedoa", "vf_dispatch_coal", "vf_dispatch_typeptr", "vf_dispatch",
     "vf_gol_neighbors", "vf_gol_swap", "vf_gen_swap", "vf_checksum_i32", "vf_launch_count", "vf_set_tuning",
     "vf_graph_bfs_init", "vf_iota_u32", "vf_fill_f32", "vf_ray_render", "vf_gol_step", "vf_gen_step",
-    "vf_dispatch_concord", "vf_micro_branch",
+    "vf_dispatch_concord", "vf_micro_branch", "vf_collide_tmp_words", "vf_collide_grid",
 ]
 APP_RAY = 4
 APP_TRAF = 5
@@ -77,6 +77,35 @@ class stut_move_args(ctypes.Structure):
 class stut_get_args(ctypes.Structure):
     _fields_ = [("vel_out_dev", ctypes.c_void_p), ("broken_out_dev", ctypes.c_void_p), ("id_base", ctypes.c_uint32),
                 ("spring_base", ctypes.c_uint32)]
+
+
+APP_COLLIDE = 8
+COLLIDE_UPDATE, COLLIDE_MERGE, COLLIDE_GET = 0, 1, 2
+
+
+class collide_update_args(ctypes.Structure):
+    _fields_ = [("P_dev", ctypes.c_void_p), ("Ps_dev", ctypes.c_void_p), ("list_dev", ctypes.c_void_p),
+                ("cell_start_dev", ctypes.c_void_p), ("Pm_dev", ctypes.c_void_p), ("Vm_dev", ctypes.c_void_p),
+                ("near_dev", ctypes.c_void_p), ("G", ctypes.c_uint32), ("rc", ctypes.c_float),
+                ("rc2", ctypes.c_float), ("rm2", ctypes.c_float), ("dt", ctypes.c_float),
+                ("eps2", ctypes.c_float * 3), ("damp", ctypes.c_float)]
+
+
+class collide_merge_args(ctypes.Structure):
+    _fields_ = [("Pm_dev", ctypes.c_void_p), ("Vm_dev", ctypes.c_void_p), ("near_dev", ctypes.c_void_p),
+                ("P_dev", ctypes.c_void_p)]
+
+
+class collide_get_args(ctypes.Structure):
+    _fields_ = [("vel_out_dev", ctypes.c_void_p), ("idx_base", ctypes.c_uint32)]
+
+
+class collide_grid_args(ctypes.Structure):
+    _fields_ = [("N", ctypes.c_uint32), ("G", ctypes.c_uint32), ("rc", ctypes.c_float),
+                ("P_dev", ctypes.c_void_p), ("cell_of_dev", ctypes.c_void_p), ("cell_count_dev", ctypes.c_void_p),
+                ("cell_start_dev", ctypes.c_void_p), ("list_dev", ctypes.c_void_p), ("Ps_dev", ctypes.c_void_p),
+                ("tmp_dev", ctypes.c_void_p), ("objs_dev", ctypes.c_void_p), ("id_lo", ctypes.c_uint32),
+                ("id_hi", ctypes.c_uint32), ("order_dev", ctypes.c_void_p), ("active_dev", ctypes.c_void_p)]
 
 
 class traf_cell_args(ctypes.Structure):
@@ -204,6 +233,8 @@ def lib(required: bool = True):
         "vf_gol_step": (I, [P, I, U32, U32, I, P, P, P, P, P, P, P]),
         "vf_dispatch_concord": (I, [P, U32, U32, P, U64, P, ctypes.c_size_t, P]),
         "vf_micro_branch": (I, [U64, U32, I, U64, U32, P, P]),
+        "vf_collide_tmp_words": (U64, [U32, U32]),
+        "vf_collide_grid": (I, [ctypes.POINTER(collide_grid_args), P]),
         "vf_gen_step": (I, [P, I, U32, U32, I, P, P, P, P, P, P, P, U32, U32, U32, P]),
     }
     for name, (res, args) in sig.items():

@@ -31,11 +31,12 @@ from paper_conf_asplos_zhangar21_b200.ray import Ray  # noqa: E402
 from paper_conf_asplos_zhangar21_b200.traf import Traf  # noqa: E402
 from paper_conf_asplos_zhangar21_b200.nbody import Nbody  # noqa: E402
 from paper_conf_asplos_zhangar21_b200.stut import Stut  # noqa: E402
+from paper_conf_asplos_zhangar21_b200.collide import Collide  # noqa: E402
 
 VARIANTS = ("cuda", "sharedoa", "coal", "typeptr")
 PEAKS = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))) if os.path.exists(
     os.path.join(ROOT, "MEASURED_PEAKS.json")) else {}
-HBM = PEAKS.get("hbm_gbs", 6550.1)
+HBM = PEAKS.get("hbm_gbs", 6650.0)  # else the B200_PROFILING.md fallback (6.65 TB/s)
 SMS = 148
 FP32_PEAK = SMS * 128 * 2 * PEAKS.get("sm_max_mhz", 1965.0) * 1e6 / 1e12  # TFLOP/s, derived
 ROWS = []
@@ -235,9 +236,33 @@ def bench_stut(ctx, quick):
         ctx.reset()
 
 
+# ---------------------------------------------------------------- config 5: collision (cutoff grid + merging)
+def bench_collide(ctx, quick):
+    N = (1 << 20) if quick else (1 << 24)
+    steps = 10
+    s = synth.collide_system(N, seed=13)
+    _, _, ocalls, sec = oracle.collide_run(s, 1, threads=oracle.max_threads())
+    cpu = cpu_info(ocalls, sec, f"full system (N={N}), 1 step")
+    # update: 8 ptr + 24 obj r + 12 obj w + 16 own P + 16 Pm w + 4 near w = 80 B; merge: 8 ptr + 24 obj r
+    # + 4 near + 16 Pm + 16 P w = 68 B; neighbour positions are L1/L2-resident
+    per_call = (80 + 68) / 2
+    for v in VARIANTS:
+        c = Collide(ctx, s, v)
+        for _ in range(2):
+            c.step()
+        torch.cuda.synchronize()
+        a0 = c.calls()
+        ms = ev_time(c.step, steps, warm=0)
+        calls = (c.calls() - a0) / steps
+        record("collide", f"N={N} bodies, cutoff grid G={s['G']}, merging", v, int(calls), ms, per_call, "GB/s",
+               "hbm", dict(objects=N), cpu)
+        del c
+        ctx.reset()
+
+
 def main():
     ap = argparse.ArgumentParser()
-    ap.add_argument("--apps", default="gol,ray,traf,gen,stut,nbody,graph")
+    ap.add_argument("--apps", default="gol,ray,traf,gen,stut,nbody,collide,graph")
     ap.add_argument("--out", default="gpurun_out/apps")
     ap.add_argument("--quick", action="store_true")
     a = ap.parse_args()
@@ -257,7 +282,7 @@ def main():
             rf = r["roofline"]
             cpu = r.get("cpu_baseline")
             f.write(f"| {r['app']} | {r['config']} | {r['variant']} | {r['calls_per_step']} | {r['ms_per_step']:.3f} | "
-                    f"{r['calls_per_s'] / 1e9:.2f} | {rel:.2f} | {rf['achieved']:.1f} {rf['unit']} | {rf['frac']:.3f} | "
+                    f"{r['calls_per_s'] / 1e9:.4g} | {rel:.2f} | {rf['achieved']:.1f} {rf['unit']} | {rf['frac']:.3f} | "
                     f"{(cpu['value'] / 1e9) if cpu else float('nan'):.3f} ({cpu['cores'] if cpu else '-'}) |\n")
     print("wrote", a.out)
 
