@@ -535,7 +535,11 @@ vf_status vf_checksum_i32(const int32_t* vals_dev, uint64_t n, long long* out_de
  * mbarrier ring in shared memory (regroup 0 only), 0 (default) uses plain
  * per-thread loads; "call" = 1 makes COAL / TYPEPTR CALL the resolved type's
  * vFunc* indirectly (the paper's design, Table 1 row C, Fig. 5b line 4), 0
- * (default) groups lanes by type and calls each body directly.
+ * (default) groups lanes by type and calls each body directly;
+ * "persistent" = 1 runs the grouped kernels on a persistent grid (CTAs loop
+ * over tiles), 0 gives every CTA one tile, -1 (default) = persistent except
+ * for the app methods marked heavy (long bodies of varying length: collision
+ * and N-body update, graph methods).
  * VF_ERR_INVALID for unknown keys / values. */
 vf_status vf_set_tuning(const char* key, int value);
 /* Number of libvf kernel launches issued since load (for bench accounting). */

@@ -181,6 +181,7 @@ struct App {
   static constexpr int kUnroll = 1;
   static constexpr int kUnrollSorted = 1;
   static constexpr int kPrefetch = 0;
+  static constexpr uint32_t kHeavyMask = 1u << VF_COLLIDE_UPDATE;  // one tile per CTA (dispatch.cuh grid_cap)
   using Base = Body;
   template <int K>
   using Type = typename TypeOf<K>::T;

@@ -199,6 +199,7 @@ struct App {
   static constexpr int kUnroll = 2;
   static constexpr int kUnrollSorted = 2;
   static constexpr int kPrefetch = 2;
+  static constexpr uint32_t kHeavyMask = 0x1Fu;  // one tile per CTA (dispatch.cuh grid_cap)
   using Base = Vertex;
   template <int K>
   using Type = VertexK<K>;

@@ -418,6 +418,9 @@ vf_status vf_set_tuning(const char* key, int value) {
   } else if (!strcmp(key, "call")) {
     if (value < 0 || value > 1) return VF_ERR_INVALID;
     tuning().call = value;
+  } else if (!strcmp(key, "persistent")) {
+    if (value < -1 || value > 1) return VF_ERR_INVALID;
+    tuning().persistent = value;
   } else {
     return VF_ERR_INVALID;
   }

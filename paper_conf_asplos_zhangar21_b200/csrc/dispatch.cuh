@@ -462,72 +462,78 @@ __global__ void __launch_bounds__(kBlock) k_dispatch_sorted(const uint64_t* __re
       }
     }
     // Tiles whose warps are already type-uniform (sorted input, run interiors)
-    // skip the sort: one barrier instead of three.
+    // skip the sort: one barrier instead of four. Both cases reach the SAME
+    // call site below (one inlined copy of each body per j: heavy bodies are
+    // not duplicated into the instruction cache).
     bool mixed = false;
 #pragma unroll
     for (int j = 0; j < U; ++j) {
       const uint32_t pres = __reduce_or_sync(0xffffffffu, t[j] < (uint32_t)App::kTypes ? (1u << t[j]) : 0u);
       mixed |= (pres & (pres - 1)) != 0;
     }
-    if (!__syncthreads_or(mixed)) {
+    const bool sorted = __syncthreads_or(mixed) != 0;  // CTA-uniform
+    if (sorted) {
+      // B: rank within type (warp-aggregated smem atomics)
 #pragma unroll
       for (int j = 0; j < U; ++j) {
-        sink ^= w[j];
-        group_call<App, M>(t[j], a[j], 0ull, base + (uint64_t)j * kBlock + threadIdx.x, args, tbl);
+        const bool ok = t[j] < (uint32_t)App::kTypes;
+        const uint32_t key = ok ? t[j] : 0xFFFFu;
+        const uint32_t peers = __match_any_sync(0xffffffffu, key);
+        const int leader = __ffs(peers) - 1;
+        uint32_t b = 0;
+        if (ok && lane == leader) b = atomicAdd(&s_hist[t[j]], (uint32_t)__popc(peers));
+        b = __shfl_sync(0xffffffffu, b, leader);
+        rank[j] = b + __popc(peers & lt_mask);
       }
-      continue;
-    }
-    // B: rank within type (warp-aggregated smem atomics)
+      __syncthreads();
+      // C: exclusive scan of the histogram (one warp), reset it for the next tile
+      if (threadIdx.x < 32) {
+        const uint32_t h = s_hist[lane];
+        uint32_t x = h;
 #pragma unroll
-    for (int j = 0; j < U; ++j) {
-      const bool ok = t[j] < (uint32_t)App::kTypes;
-      const uint32_t key = ok ? t[j] : 0xFFFFu;
-      const uint32_t peers = __match_any_sync(0xffffffffu, key);
-      const int leader = __ffs(peers) - 1;
-      uint32_t b = 0;
-      if (ok && lane == leader) b = atomicAdd(&s_hist[t[j]], (uint32_t)__popc(peers));
-      b = __shfl_sync(0xffffffffu, b, leader);
-      rank[j] = b + __popc(peers & lt_mask);
-    }
-    __syncthreads();
-    // C: exclusive scan of the histogram (one warp), reset it for the next tile
-    if (threadIdx.x < 32) {
-      const uint32_t h = s_hist[lane];
-      uint32_t x = h;
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
-        if (lane >= o) x += y;
+        for (int o = 1; o < 32; o <<= 1) {
+          const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+          if (lane >= o) x += y;
+        }
+        s_offs[lane] = x - h;
+        if (lane == 31) s_offs[32] = x;
+        s_hist[lane] = 0;
       }
-      s_offs[lane] = x - h;
-      if (lane == 31) s_offs[32] = x;
-      s_hist[lane] = 0;
-    }
-    __syncthreads();
-    // D: scatter into the sorted tile
+      __syncthreads();
+      // D: scatter into the sorted tile
 #pragma unroll
-    for (int j = 0; j < U; ++j) {
-      if (t[j] < (uint32_t)App::kTypes) {
-        const uint32_t pos = s_offs[t[j]] + rank[j];
-        s_a[pos] = a[j];
-        s_i[pos] = (uint32_t)(j * kBlock + threadIdx.x);
-        s_t[pos] = (uint8_t)t[j];
+      for (int j = 0; j < U; ++j) {
+        if (t[j] < (uint32_t)App::kTypes) {
+          const uint32_t pos = s_offs[t[j]] + rank[j];
+          s_a[pos] = a[j];
+          s_i[pos] = (uint32_t)(j * kBlock + threadIdx.x);
+          s_t[pos] = (uint8_t)t[j];
+        }
       }
+      __syncthreads();
     }
-    __syncthreads();
-    // E: each warp walks 32 consecutive sorted entries per j
-    const uint32_t total = s_offs[32];
+    // E: each warp walks 32 consecutive (sorted) entries per j
+    const uint32_t total = sorted ? s_offs[32] : 0u;
 #pragma unroll
     for (int j = 0; j < U; ++j) sink ^= w[j];
 #pragma unroll
     for (int j = 0; j < U; ++j) {
-      const uint32_t e = (uint32_t)(j * kBlock) + threadIdx.x;
-      const bool v = e < total;
-      const uint64_t ae = v ? s_a[e] : 0ull;
-      const uint32_t te = v ? (uint32_t)s_t[e] : kNF;
-      const uint64_t ie = v ? base + s_i[e] : 0ull;
+      uint64_t ae, ie;
+      uint32_t te;
+      if (sorted) {
+        const uint32_t e = (uint32_t)(j * kBlock) + threadIdx.x;
+        const bool v = e < total;
+        ae = v ? s_a[e] : 0ull;
+        te = v ? (uint32_t)s_t[e] : kNF;
+        ie = v ? base + s_i[e] : 0ull;
+      } else {
+        ae = a[j];
+        te = t[j];
+        ie = base + (uint64_t)j * kBlock + threadIdx.x;
+      }
       group_call<App, M>(te, ae, 0ull, ie, args, tbl);
     }
+    // (the next tile's __syncthreads_or orders these reads before its scatter)
   }
   if constexpr (PF == 2) {
     if (sink == 0x8BADF00Du && n == ~0ull) asm volatile("st.global.u32 [%0], %1;" ::"l"(objs), "r"(sink));
@@ -758,6 +764,26 @@ inline unsigned grid_for(uint64_t n, uint64_t per_block, uint64_t cap) {
   return (unsigned)g;
 }
 
+// Persistent grid (occupancy x SMs, CTAs loop over tiles) or one tile per CTA.
+// Apps may mark methods whose bodies are long and of varying length
+// (kHeavyMask bit M): there a persistent CTA would wait at every tile's
+// barrier for its slowest warp, while one tile per CTA lets finished warps
+// leave and other CTAs take their place. Tuning key "persistent" overrides.
+template <class A, class = void>
+struct HeavyMask {
+  static constexpr uint32_t value = 0;
+};
+template <class A>
+struct HeavyMask<A, std::void_t<decltype(A::kHeavyMask)>> {
+  static constexpr uint32_t value = A::kHeavyMask;
+};
+template <class App, int M>
+inline uint64_t grid_cap(int occ) {
+  const int p = tuning().persistent;
+  const bool pers = p >= 0 ? p != 0 : ((HeavyMask<App>::value >> M) & 1u) == 0;
+  return pers ? (uint64_t)num_sms() * occ : ~0ull;
+}
+
 template <class App, int M, class R, int U, int PF>
 cudaError_t launch_grouped(const uint64_t* objs, uint64_t n, const ArgBlob& args,
                            const DevTable& tbl, cudaStream_t s) {
@@ -772,7 +798,7 @@ cudaError_t launch_grouped(const uint64_t* objs, uint64_t n, const ArgBlob& args
     if (occ < 1) occ = 1;
     occ_sm = sm;
   }
-  const unsigned grid = grid_for(n, (uint64_t)kBlock * U, (uint64_t)num_sms() * occ);
+  const unsigned grid = grid_for(n, (uint64_t)kBlock * U, grid_cap<App, M>(occ));
   kern<<<grid, kBlock, sm, s>>>(objs, n, args, tbl);
   note_launch();
   return cudaGetLastError();
@@ -823,7 +849,7 @@ cudaError_t launch_sorted(const uint64_t* objs, uint64_t n, const ArgBlob& args,
     if (occ < 1) occ = 1;
     occ_sm = sm;
   }
-  const unsigned grid = grid_for(n, (uint64_t)kBlock * U, (uint64_t)num_sms() * occ);
+  const unsigned grid = grid_for(n, (uint64_t)kBlock * U, grid_cap<App, M>(occ));
   kern<<<grid, kBlock, sm, s>>>(objs, n, args, tbl);
   note_launch();
   return cudaGetLastError();

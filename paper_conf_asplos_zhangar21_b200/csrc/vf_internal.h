@@ -87,6 +87,7 @@ struct Tuning {
   int pipeline = 0;   // 1: TMA-pipelined pointer stream (k_dispatch_pipe), 0: plain loads
   int regroup = 1;    // 1: CTA-level counting sort of each tile by type (k_dispatch_sorted)
   int call = 0;       // COAL / TypePointer: 0 grouped direct call, 1 indirect CALL via vFunc* table
+  int persistent = -1; // grouped kernels: 1 persistent grid, 0 one tile per CTA, -1 app default (kHeavyMask)
 };
 Tuning& tuning();
 

@@ -129,9 +129,10 @@ class Graph:
             self.ctx._check(st, f"graph method {method}")
 
     # ---------------------------------------------------------------- BFS
-    def bfs(self, src: int, mode: str = "topdown"):
+    def bfs(self, src: int, mode: str = "topdown", alpha: int = 64):
         """Level-synchronous BFS from src; returns (depth tensor, levels, calls).
         topdown: one virtual bfs_expand() per frontier work entry (single GPU);
+        hybrid: top-down, then bottom-up once the frontier exceeds V / alpha entries (single GPU);
         bottomup: one virtual bfs_probe() per owned work entry per level (multi-GPU)."""
         L = vf.lib()
         st = L.vf_graph_bfs_init(self.V, self.depth.data_ptr(), src, self.vobj.data_ptr(), self.offs.data_ptr(),
@@ -140,7 +141,32 @@ class Graph:
         if st:
             raise vf.VFError(st, "bfs_init")
         calls, level = 0, 0
-        if mode == "topdown" and self.world == 1:
+        if mode == "hybrid" and self.world == 1:
+            # direction-optimizing (Beamer): top-down while the frontier is small,
+            # bottom-up probes over every entry once it holds > V / alpha entries
+            # (depths are unique, reading G23, so the result is the same)
+            n = _sync_scalar(self.count)
+            while n > 0 and n <= self.V // alpha:
+                self.count.zero_()
+                a = vf.graph_bfs_args(self.offs.data_ptr(), self.col.data_ptr(), self.depth.data_ptr(),
+                                      self.vobj.data_ptr(), self.qc[0].data_ptr(), self.q[1].data_ptr(),
+                                      self.qc[1].data_ptr(), self.count.data_ptr(), level, self.C)
+                self._dispatch(vf.GRAPH_BFS_EXPAND, self.q[0].data_ptr(), n, a)
+                calls += n
+                n = _sync_scalar(self.count)
+                self.q[0], self.q[1] = self.q[1], self.q[0]
+                self.qc[0], self.qc[1] = self.qc[1], self.qc[0]
+                level += 1
+            while n > 0:
+                self.count.zero_()
+                a = vf.graph_bfs_args(self.offs.data_ptr(), self.col.data_ptr(), self.depth.data_ptr(),
+                                      self.vobj.data_ptr(), self.entry_chunk.data_ptr(), 0, 0, self.count.data_ptr(),
+                                      level, self.C)
+                self._dispatch(vf.GRAPH_BFS_PROBE, self.entries.data_ptr(), self.E, a)
+                calls += self.E
+                n = _sync_scalar(self.count)
+                level += 1
+        elif mode == "topdown" and self.world == 1:
             n = _sync_scalar(self.count)
             while n > 0:
                 self.count.zero_()

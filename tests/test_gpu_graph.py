@@ -49,6 +49,9 @@ def test_graph_parity(ctx, rmat, variant, chunk):
     assert levels == rmat["levels"] and int((d >= 0).sum()) == rmat["calls"] and calls >= rmat["calls"]
     d2, _, _ = g.bfs(rmat["src"], mode="bottomup")
     assert np.array_equal(d2.cpu().numpy(), rmat["depth"])
+    for alpha in (1 << 30, 64, 1):  # bottom-up at once / switch mid-way / never
+        d3, lv3, _ = g.bfs(rmat["src"], mode="hybrid", alpha=alpha)
+        assert np.array_equal(d3.cpu().numpy(), rmat["depth"]) and lv3 == rmat["levels"]
     label, iters, _ = g.cc()
     assert np.array_equal(label.cpu().numpy().view(np.uint32), rmat["label"])
     assert iters == rmat["iters"]

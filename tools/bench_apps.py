@@ -145,6 +145,11 @@ def bench_graph(ctx, quick):
         # per reached vertex: 8 B ptr + 8 B offs + per arc 4 B col + 4 B depth
         record("graph-bfs", f"rmat-{scale} top-down BFS from max-degree vertex", v, calls, ms,
                16 + 8 * avg_deg, "GB/s", "hbm", dict(V=V, arcs=arcs), cpu["bfs"])
+        ms = ev_time(lambda: g.bfs(src, mode="hybrid"), 3, warm=1)
+        # bottom-up levels dispatch every entry (visited ones return after the 8 B ptr + 16 B object read)
+        record("graph-bfs-hybrid", f"rmat-{scale} direction-optimizing BFS (top-down, then bottom-up probes)", v,
+               g.calls, ms, 16 + 8 * avg_deg * bcalls / max(g.calls, 1), "GB/s", "hbm", dict(V=V, arcs=arcs),
+               cpu["bfs"])
         ms = ev_time(lambda: g.cc(), 2, warm=1)
         record("graph-cc", f"rmat-{scale} Jacobi CC to convergence", v, g.calls, ms, 20 + 8 * avg_deg, "GB/s",
                "hbm", dict(iters=g.calls // V), cpu["cc"])
@@ -265,7 +270,11 @@ def main():
     ap.add_argument("--apps", default="gol,ray,traf,gen,stut,nbody,collide,graph")
     ap.add_argument("--out", default="gpurun_out/apps")
     ap.add_argument("--quick", action="store_true")
+    ap.add_argument("--tune", action="append", default=[], help="libvf tuning knob key=value (vf_set_tuning)")
     a = ap.parse_args()
+    for kv in a.tune:
+        k, v = kv.split("=")
+        vf.set_tuning(k, int(v))
     ctx = vf.Ctx(0, cuda_heap_bytes=16 << 30)
     for name in a.apps.split(","):
         globals()[f"bench_{name}"](ctx, a.quick)

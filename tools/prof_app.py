@@ -51,6 +51,11 @@ def main():
         nb = Nbody(ctx, synth.nbody_system(65536, seed=10), a.variant)
         for _ in range(a.steps):
             nb.step()
+    elif a.app == "collide":
+        from paper_conf_asplos_zhangar21_b200.collide import Collide
+        c = Collide(ctx, synth.collide_system(1 << 24, seed=13), a.variant)
+        for _ in range(a.steps):
+            c.step()
     elif a.app == "traf":
         from paper_conf_asplos_zhangar21_b200.traf import Traf
         t = Traf(ctx, synth.traf_world(3277, 4096, seed=11), a.variant)
