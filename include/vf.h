@@ -165,6 +165,7 @@ typedef struct {
   const float4_t* Ps_dev;          /* N, cell-sorted copy: Ps[e] = P[list[e]]          */
   const uint32_t* list_dev;        /* ids in cell order, ascending within a cell       */
   const uint32_t* cell_start_dev;  /* G^3 + 1 offsets into list                         */
+  const uint32_t* slot_dev;        /* N, slot[id] = e with list[e] = id (active bodies) */
   float4_t* Pm_dev;                /* N, post-update position + mass, by id             */
   float4_t* Vm_dev;                /* N, post-update velocity (written when near >= 0)  */
   int32_t* near_dev;               /* N, nearest body within rm or -1                   */
@@ -478,7 +479,7 @@ vf_status vf_ray_render(vf_ctx* ctx, vf_variant v, const uint64_t* shapes_dev, u
  * For every body i with P[i].w > 0: cell (clamp(floor(x/rc)), clamp(floor(y/rc)),
  * clamp(floor(z/rc))) of a G^3 grid, c = (z*G + y)*G + x; cell_start = the
  * exclusive prefix sum of the cell counts; list[cell_start[c] ..) = the ids of
- * cell c ascending; Ps[e] = P[list[e]]. Then order[k] = the objects of the
+ * cell c ascending; Ps[e] = P[list[e]]; slot[list[e]] = e. Then order[k] = the objects of the
  * owned ids [id_lo, id_hi) that are active, in cell order (spatially
  * neighbouring bodies share a warp), null-padded to id_hi - id_lo entries
  * (null pointers are skipped by every dispatch variant). *active_dev (if not
@@ -495,6 +496,7 @@ typedef struct {
   uint32_t* cell_start_dev;       /* G^3 + 1                                    */
   uint32_t* list_dev;             /* N                                          */
   float4_t* Ps_dev;               /* N                                          */
+  uint32_t* slot_dev;             /* N (entries of inactive bodies untouched)   */
   uint32_t* tmp_dev;              /* vf_collide_tmp_words(N, G)                 */
   const uint64_t* objs_dev;       /* id_hi - id_lo: object of body id_lo + k     */
   uint32_t id_lo, id_hi;

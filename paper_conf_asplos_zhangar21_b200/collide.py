@@ -56,6 +56,7 @@ class Collide:
         self.cell_count = torch.zeros(ncell, **u32)
         self.cell_start = torch.zeros(ncell + 1, **u32)
         self.list = torch.zeros(max(N, 1), **u32)
+        self.slot = torch.zeros(max(N, 1), **u32)
         self.tmp = torch.zeros(int(vf.lib().vf_collide_tmp_words(N, self.G)), **u32)
         self.order = torch.zeros(max(self.hi - self.lo, 1), dtype=torch.int64, device=dev)
         self.active = torch.zeros(1, dtype=torch.int64, device=dev)  # owned active bodies, summed over steps
@@ -65,12 +66,13 @@ class Collide:
         self.eps2 = [float(x) for x in sys_["eps2"]]
         self._grid = vf.collide_grid_args(
             N, self.G, self.rc, self.P.data_ptr(), self.cell_of.data_ptr(), self.cell_count.data_ptr(),
-            self.cell_start.data_ptr(), self.list.data_ptr(), self.Ps.data_ptr(), self.tmp.data_ptr(),
+            self.cell_start.data_ptr(), self.list.data_ptr(), self.Ps.data_ptr(), self.slot.data_ptr(),
+            self.tmp.data_ptr(),
             self.objs.data_ptr() if self.hi > self.lo else None, self.lo, self.hi, self.order.data_ptr(),
             self.active.data_ptr())
         self._upd = vf.collide_update_args(
             self.P.data_ptr(), self.Ps.data_ptr(), self.list.data_ptr(), self.cell_start.data_ptr(),
-            self.Pm.data_ptr(), self.Vm.data_ptr(), self.near.data_ptr(), self.G, self.rc, self.rc2, self.rm2,
+            self.slot.data_ptr(), self.Pm.data_ptr(), self.Vm.data_ptr(), self.near.data_ptr(), self.G, self.rc, self.rc2, self.rm2,
             self.dt, (ctypes.c_float * 3)(*self.eps2), self.damp)
         self._mrg = vf.collide_merge_args(self.Pm.data_ptr(), self.Vm.data_ptr(), self.near.data_ptr(),
                                           self.P.data_ptr())

@@ -52,9 +52,14 @@ struct Body {
   // three cells x-1, x, x+1 of one (z, y) row are consecutive in the cell
   // index, so their bodies are ONE contiguous run of list / Ps in exactly the
   // oracle's order (x ascending, ids ascending within a cell): 9 runs per body.
+  // "j != me" compares slots (slot[me]), so the id array is read only for
+  // candidates within rm. (Measured on B200: batching 4 candidates for ILP,
+  // with or without a predicated force term, raises registers 48 -> 71 and
+  // costs occupancy: 1.6x slower.)
   __device__ __forceinline__ void update_with(const vf_collide_update_args& a, float eps2, bool damped) {
     const uint32_t me = idx;
     const float4 pi = __ldg(a.P_dev + me);
+    const uint32_t es = __ldg(a.slot_dev + me);
     const int G = (int)a.G;
     const int cx = cell_coord(pi.x, a.rc, G), cy = cell_coord(pi.y, a.rc, G), cz = cell_coord(pi.z, a.rc, G);
     const int x0 = cx > 0 ? cx - 1 : 0, x1 = cx + 1 < G ? cx + 1 : G - 1;
@@ -71,22 +76,23 @@ struct Body {
         const uint32_t e1 = __ldg(a.cell_start_dev + row + x1 + 1);
 #pragma unroll 2
         for (uint32_t e = e0; e < e1; ++e) {
-          const uint32_t j = __ldg(a.list_dev + e);
           const float4 pj = __ldg(a.Ps_dev + e);
           const float dx = pj.x - pi.x, dy = pj.y - pi.y, dz = pj.z - pi.z;
           const float d2 = fmaf(dx, dx, fmaf(dy, dy, dz * dz));
-          const bool other = j != me;
-          if (other && d2 < rc2) {
+          const bool other = e != es;
+          if (other && d2 < rc2) {  // ~1 candidate in 6 (sphere / 27 cells)
             const float r2 = fmaf(dx, dx, fmaf(dy, dy, fmaf(dz, dz, eps2)));
-            const float inv = rcp_rn_fast(r2 * sqrt_rn_fast(r2));  // == 1.0f / (r2 * sqrtf(r2))
-            const float sc = pj.w * inv;
+            const float sc = pj.w * rcp_rn_fast(r2 * sqrt_rn_fast(r2));  // m_j * (1.0f / (r2 * sqrtf(r2)))
             ax = fmaf(dx, sc, ax);
             ay = fmaf(dy, sc, ay);
             az = fmaf(dz, sc, az);
           }
-          if (other && d2 < rm2 && (bestj < 0 || d2 < best || (d2 == best && (int32_t)j < bestj))) {
-            best = d2;
-            bestj = (int32_t)j;
+          if (other && d2 < rm2 && (bestj < 0 || d2 <= best)) {  // rare: read the id
+            const int32_t j = (int32_t)__ldg(a.list_dev + e);
+            if (bestj < 0 || d2 < best || j < bestj) {
+              best = d2;
+              bestj = j;
+            }
           }
         }
       }
@@ -182,6 +188,7 @@ struct App {
   static constexpr int kUnrollSorted = 1;
   static constexpr int kPrefetch = 0;
   static constexpr uint32_t kHeavyMask = 1u << VF_COLLIDE_UPDATE;  // one tile per CTA (dispatch.cuh grid_cap)
+  static constexpr int kMinBlocks = 5;  // <= 48 registers: 40 warps per SM hide the gather latency
   using Base = Body;
   template <int K>
   using Type = typename TypeOf<K>::T;
@@ -328,7 +335,7 @@ __global__ void k_fill(uint32_t N, const uint32_t* __restrict__ cell_of, uint32_
 
 // per cell: ids ascending (insertion sort; ~per_cell entries), then Ps
 __global__ void k_sort_cells(uint32_t ncell, const uint32_t* __restrict__ start, uint32_t* __restrict__ list,
-                             const float4* __restrict__ P, float4* __restrict__ Ps) {
+                             const float4* __restrict__ P, float4* __restrict__ Ps, uint32_t* __restrict__ slot) {
   const uint32_t stride = gridDim.x * blockDim.x;
   for (uint32_t c = blockIdx.x * blockDim.x + threadIdx.x; c < ncell; c += stride) {
     const uint32_t s = start[c], e = start[c + 1];
@@ -341,7 +348,11 @@ __global__ void k_sort_cells(uint32_t ncell, const uint32_t* __restrict__ start,
       }
       list[m] = x;
     }
-    for (uint32_t k = s; k < e; ++k) Ps[k] = __ldg(P + list[k]);
+    for (uint32_t k = s; k < e; ++k) {
+      const uint32_t id = list[k];
+      Ps[k] = __ldg(P + id);
+      slot[id] = k;
+    }
   }
 }
 
@@ -421,7 +432,7 @@ extern "C" uint64_t vf_collide_tmp_words(uint32_t N, uint32_t G) {
 extern "C" vf_status vf_collide_grid(const vf_collide_grid_args* a, void* stream) {
   if (!a || a->G < 1 || a->G > 1024 || !(a->rc > 0.0f) || a->id_lo > a->id_hi || a->id_hi > a->N) return VF_ERR_INVALID;
   if (a->N && (!a->P_dev || !a->cell_of_dev || !a->cell_count_dev || !a->cell_start_dev || !a->list_dev ||
-               !a->Ps_dev || !a->tmp_dev))
+               !a->Ps_dev || !a->slot_dev || !a->tmp_dev))
     return VF_ERR_INVALID;
   if (a->id_hi > a->id_lo && (!a->objs_dev || !a->order_dev)) return VF_ERR_INVALID;
   const cudaStream_t s = (cudaStream_t)stream;
@@ -440,7 +451,8 @@ extern "C" vf_status vf_collide_grid(const vf_collide_grid_args* a, void* stream
   if (e != cudaSuccess) return VF_ERR_CUDA;
   if (N) {
     k_fill<<<grid, 256, 0, s>>>(N, a->cell_of_dev, a->cell_count_dev, a->cell_start_dev, a->list_dev);
-    k_sort_cells<<<grid, 256, 0, s>>>((uint32_t)ncell, a->cell_start_dev, a->list_dev, a->P_dev, a->Ps_dev);
+    k_sort_cells<<<grid, 256, 0, s>>>((uint32_t)ncell, a->cell_start_dev, a->list_dev, a->P_dev, a->Ps_dev,
+                                        a->slot_dev);
     vf::note_launch(2);
   }
   const uint32_t* total = a->cell_start_dev + ncell;

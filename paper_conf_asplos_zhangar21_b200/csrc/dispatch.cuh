@@ -38,6 +38,18 @@ __device__ __forceinline__ T blob_as(const ArgBlob& b) {
   return *reinterpret_cast<const T*>(b.b);
 }
 
+// Minimum resident CTAs per SM the dispatch kernels are compiled for
+// (__launch_bounds__ min blocks; caps registers). Apps whose bodies keep many
+// values in flight set kMinBlocks so the whole grid stays resident.
+template <class A, class = void>
+struct MinBlocks {
+  static constexpr int value = 1;
+};
+template <class A>
+struct MinBlocks<A, std::void_t<decltype(A::kMinBlocks)>> {
+  static constexpr int value = A::kMinBlocks;
+};
+
 __device__ __forceinline__ uint64_t ldg_u64(const uint64_t* p) {
   uint64_t v;
   asm volatile("ld.global.nc.L1::no_allocate.u64 %0, [%1];" : "=l"(v) : "l"(p));
@@ -190,7 +202,7 @@ __device__ __forceinline__ void warm_line(uint64_t a, uint32_t& sink) {
 // tiles of kBlock*U objects; every lane of every warp runs the same number of
 // iterations, so the full-mask warp collectives are legal.
 template <class App, int M, class R, int U, int PF>
-__global__ void __launch_bounds__(kBlock) k_dispatch_grouped(const uint64_t* __restrict__ objs,
+__global__ void __launch_bounds__(kBlock, MinBlocks<App>::value) k_dispatch_grouped(const uint64_t* __restrict__ objs,
                                                              uint64_t n, ArgBlob args,
                                                              DevTable tbl) {
   extern __shared__ __align__(16) unsigned char smem[];
@@ -419,7 +431,7 @@ struct SortSmem {
 };
 
 template <class App, int M, class R, int U, int PF>
-__global__ void __launch_bounds__(kBlock) k_dispatch_sorted(const uint64_t* __restrict__ objs,
+__global__ void __launch_bounds__(kBlock, MinBlocks<App>::value) k_dispatch_sorted(const uint64_t* __restrict__ objs,
                                                             uint64_t n, ArgBlob args, DevTable tbl) {
   static_assert(App::kTypes <= 32, "one warp scans the histogram");
   extern __shared__ __align__(16) unsigned char smem[];
@@ -609,7 +621,7 @@ __device__ __forceinline__ void fill_thunks(ThunkFn* tab) {
 }
 
 template <class App, int M, class R>
-__global__ void __launch_bounds__(kBlock) k_dispatch_indirect(const uint64_t* __restrict__ objs, uint64_t n,
+__global__ void __launch_bounds__(kBlock, MinBlocks<App>::value) k_dispatch_indirect(const uint64_t* __restrict__ objs, uint64_t n,
                                                                ArgBlob args, DevTable tbl) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ ThunkFn s_fn[App::kTypes];
@@ -638,7 +650,7 @@ __global__ void __launch_bounds__(kBlock) k_dispatch_indirect(const uint64_t* __
 // CUDA / SharedOA dispatch: the plain C++ virtual call, one object per thread,
 // as the user writes it (`objs[i]->f()`).
 template <class App, int M>
-__global__ void __launch_bounds__(kBlock) k_dispatch_virtual(const uint64_t* __restrict__ objs,
+__global__ void __launch_bounds__(kBlock, MinBlocks<App>::value) k_dispatch_virtual(const uint64_t* __restrict__ objs,
                                                              uint64_t n, ArgBlob args) {
   const uint64_t i = (uint64_t)blockIdx.x * kBlock + threadIdx.x;
   if (i < n) {

@@ -85,7 +85,8 @@ COLLIDE_UPDATE, COLLIDE_MERGE, COLLIDE_GET = 0, 1, 2
 
 class collide_update_args(ctypes.Structure):
     _fields_ = [("P_dev", ctypes.c_void_p), ("Ps_dev", ctypes.c_void_p), ("list_dev", ctypes.c_void_p),
-                ("cell_start_dev", ctypes.c_void_p), ("Pm_dev", ctypes.c_void_p), ("Vm_dev", ctypes.c_void_p),
+                ("cell_start_dev", ctypes.c_void_p), ("slot_dev", ctypes.c_void_p), ("Pm_dev", ctypes.c_void_p),
+                ("Vm_dev", ctypes.c_void_p),
                 ("near_dev", ctypes.c_void_p), ("G", ctypes.c_uint32), ("rc", ctypes.c_float),
                 ("rc2", ctypes.c_float), ("rm2", ctypes.c_float), ("dt", ctypes.c_float),
                 ("eps2", ctypes.c_float * 3), ("damp", ctypes.c_float)]
@@ -104,7 +105,7 @@ class collide_grid_args(ctypes.Structure):
     _fields_ = [("N", ctypes.c_uint32), ("G", ctypes.c_uint32), ("rc", ctypes.c_float),
                 ("P_dev", ctypes.c_void_p), ("cell_of_dev", ctypes.c_void_p), ("cell_count_dev", ctypes.c_void_p),
                 ("cell_start_dev", ctypes.c_void_p), ("list_dev", ctypes.c_void_p), ("Ps_dev", ctypes.c_void_p),
-                ("tmp_dev", ctypes.c_void_p), ("objs_dev", ctypes.c_void_p), ("id_lo", ctypes.c_uint32),
+                ("slot_dev", ctypes.c_void_p), ("tmp_dev", ctypes.c_void_p), ("objs_dev", ctypes.c_void_p), ("id_lo", ctypes.c_uint32),
                 ("id_hi", ctypes.c_uint32), ("order_dev", ctypes.c_void_p), ("active_dev", ctypes.c_void_p)]
 
 
