@@ -27,7 +27,7 @@ import numpy as np
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 SO = os.path.join(HERE, "liboracle.so")
-SOURCES = ["alloc.cpp", "micro.cpp", "gol.cpp", "gen.cpp", "graph.cpp", "ray.cpp", "traf.cpp", "nbody.cpp", "stut.cpp", "collide.cpp"]
+SOURCES = ["alloc.cpp", "micro.cpp", "gol.cpp", "gen.cpp", "graph.cpp", "graph_en.cpp", "ray.cpp", "traf.cpp", "nbody.cpp", "stut.cpp", "collide.cpp"]
 NOT_FOUND = 0xFFFFFFFF
 
 
@@ -86,6 +86,14 @@ def lib():
         L.oracle_graph_bfs.argtypes = [U64, P, P, P, U32, P, P, P, ctypes.POINTER(ctypes.c_double)]
         L.oracle_graph_cc.restype = ctypes.c_int
         L.oracle_graph_cc.argtypes = [U64, P, P, P, ctypes.c_int, P, P, P, ctypes.POINTER(ctypes.c_double)]
+        L.oracle_graph_en_edge_types.restype = ctypes.c_int
+        L.oracle_graph_en_edge_types.argtypes = [U64, P, P, P]
+        L.oracle_graph_en_bfs.restype = ctypes.c_int
+        L.oracle_graph_en_bfs.argtypes = [U64, P, P, P, U32, P, P, P, P, ctypes.POINTER(ctypes.c_double)]
+        L.oracle_graph_en_cc.restype = ctypes.c_int
+        L.oracle_graph_en_cc.argtypes = [U64, P, P, P, P, P, P, P, ctypes.POINTER(ctypes.c_double)]
+        L.oracle_graph_en_pr.restype = ctypes.c_int
+        L.oracle_graph_en_pr.argtypes = [U64, P, P, P, ctypes.c_double, U32, P, ctypes.POINTER(ctypes.c_double)]
         L.oracle_graph_pr.restype = ctypes.c_int
         L.oracle_graph_pr.argtypes = [U64, P, P, P, ctypes.c_double, U32, ctypes.c_int, P,
                                       ctypes.POINTER(ctypes.c_double)]
@@ -261,6 +269,55 @@ def graph_pr(offs, col, types, iters: int = 20, d: float = 0.85, threads: int = 
                                rank.ctypes.data, ctypes.byref(sec))
     if rc:
         raise ValueError(f"oracle_graph_pr rc={rc}")
+    return rank, sec.value
+
+
+def graph_en_edge_types(offs, vtypes):
+    """GraphChi-vEN edge class of every arc (0 Edge, 1 HubEdge: source is a Hub)."""
+    offs = np.ascontiguousarray(offs, dtype=np.uint64)
+    vtypes = np.ascontiguousarray(vtypes, dtype=np.uint32)
+    V = len(offs) - 1
+    et = np.empty(int(offs[-1]), np.uint32)
+    lib().oracle_graph_en_edge_types(V, offs.ctypes.data, vtypes.ctypes.data, et.ctypes.data)
+    return et
+
+
+def graph_en_bfs(offs, col, types, src: int):
+    """Virtual edges + vertices. Returns (depth int32[V], levels, vertex calls, edge calls, seconds)."""
+    offs, col, types = _csr(offs, col, types)
+    V = len(offs) - 1
+    depth = np.empty(V, np.int32)
+    lv, vc, ec, sec = ctypes.c_uint32(), ctypes.c_uint64(), ctypes.c_uint64(), ctypes.c_double()
+    rc = lib().oracle_graph_en_bfs(V, offs.ctypes.data, col.ctypes.data, types.ctypes.data, src, depth.ctypes.data,
+                                   ctypes.byref(lv), ctypes.byref(vc), ctypes.byref(ec), ctypes.byref(sec))
+    if rc:
+        raise ValueError(f"oracle_graph_en_bfs rc={rc}")
+    return depth, lv.value, vc.value, ec.value, sec.value
+
+
+def graph_en_cc(offs, col, types):
+    """Virtual edges + vertices. Returns (label uint32[V], iters, vertex calls, edge calls, seconds)."""
+    offs, col, types = _csr(offs, col, types)
+    V = len(offs) - 1
+    label = np.empty(V, np.uint32)
+    it, vc, ec, sec = ctypes.c_uint32(), ctypes.c_uint64(), ctypes.c_uint64(), ctypes.c_double()
+    rc = lib().oracle_graph_en_cc(V, offs.ctypes.data, col.ctypes.data, types.ctypes.data, label.ctypes.data,
+                                  ctypes.byref(it), ctypes.byref(vc), ctypes.byref(ec), ctypes.byref(sec))
+    if rc:
+        raise ValueError(f"oracle_graph_en_cc rc={rc}")
+    return label, it.value, vc.value, ec.value, sec.value
+
+
+def graph_en_pr(offs, col, types, iters: int = 20, d: float = 0.85):
+    """Virtual edges + vertices. Returns (rank float32[V], seconds)."""
+    offs, col, types = _csr(offs, col, types)
+    V = len(offs) - 1
+    rank = np.empty(V, np.float32)
+    sec = ctypes.c_double()
+    rc = lib().oracle_graph_en_pr(V, offs.ctypes.data, col.ctypes.data, types.ctypes.data, d, iters,
+                                  rank.ctypes.data, ctypes.byref(sec))
+    if rc:
+        raise ValueError(f"oracle_graph_en_pr rc={rc}")
     return rank, sec.value
 
 

@@ -122,6 +122,31 @@ int oracle_graph_cc(uint64_t V, const uint64_t* offs, const uint32_t* col, const
 int oracle_graph_pr(uint64_t V, const uint64_t* offs, const uint32_t* col, const uint32_t* types,
                     double d, uint32_t iters, int threads, float* rank, double* seconds);
 
+/* ---- GraphChi-vEN: virtual edges AND virtual vertices (Table 2
+ * P:1566-1588; readings G32/G33). One edge object per arc
+ * (u -> v) from plain `new` in arc order (ChiEdge / Edge / HubEdge: HubEdge
+ * iff the source is a Hub, etypes[k] = 1), double-buffered value; per vertex
+ * in-edge list (arcs (u -> v), ascending u) and out-edge list (own arcs).
+ * BFS: as oracle_graph_bfs, each vertex visits its out-edges through the
+ *   virtual target(); *vcalls = vertex calls, *ecalls = edge calls.
+ * CC: edges start with their source's label; update(v): m = min(label_in[v],
+ *   virtual get_label(b) over in-edges), label_out[v] = m, virtual
+ *   set_label(1-b, m) on out-edges; until no change. Same labels as
+ *   oracle_graph_cc.
+ * PR: edges start with r0(u)/deg(u); update(v): s = sum of virtual get_pr(b)
+ *   over in-edges (ascending u), r' = (float)((1-d)/V + d*(s + D/V)), virtual
+ *   set_pr(1-b, r'/deg) on out-edges; D of the next iteration = sum of r'
+ *   over deg-0 vertices in vertex order. Bit-identical to oracle_graph_pr. */
+int oracle_graph_en_edge_types(uint64_t V, const uint64_t* offs, const uint32_t* vtypes, uint32_t* etypes);
+int oracle_graph_en_bfs(uint64_t V, const uint64_t* offs, const uint32_t* col, const uint32_t* types,
+                        uint32_t src, int32_t* depth, uint32_t* levels, uint64_t* vcalls,
+                        uint64_t* ecalls, double* seconds);
+int oracle_graph_en_cc(uint64_t V, const uint64_t* offs, const uint32_t* col, const uint32_t* types,
+                       uint32_t* label, uint32_t* iters, uint64_t* vcalls, uint64_t* ecalls,
+                       double* seconds);
+int oracle_graph_en_pr(uint64_t V, const uint64_t* offs, const uint32_t* col, const uint32_t* types,
+                       double d, uint32_t iters, float* rank, double* seconds);
+
 /* ---- Config 3 ray tracer over polymorphic shapes (Table 2 RAY P:1592-1600;
  * readings G24, G25). Shapes j = 0..S-1 of type types[j] (0 Plane y=h,
  * 1 Sphere, 2 axis-aligned Rect, 3 Triangle) with 12 fp32 params each
