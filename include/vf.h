@@ -83,7 +83,9 @@ enum {
   VF_APP_NBODY = 6, /* config 5: Body / Star / Planet / Dust (all-pairs N-body, G18)      */
   VF_APP_STUT = 7,  /* config 5: Element / Node / AnchorNode / AnchorPullNode / Spring   */
   VF_APP_COLLIDE = 8, /* config 5: Body / Star / Planet / Dust (cutoff grid + merging, G19) */
-  VF_APP_COUNT = 9
+  VF_APP_GRAPH_EN = 9,/* GraphChi-vEN vertices: ChiVertex / Leaf / Low / Mid / Hub */
+  VF_APP_EDGE = 10,   /* GraphChi-vEN edges: ChiEdge / Edge / HubEdge  (G32)     */
+  VF_APP_COUNT = 11
 };
 
 /* Methods of VF_APP_STUT (Table 2 "structure" P:1524-1528, reading G17). Type
@@ -306,6 +308,106 @@ typedef struct {
   uint32_t* counter_dev;       /* per vertex, zero between iterations              */
   uint32_t C;
 } vf_graph_pr_args;
+
+/* GraphChi-vEN: virtual edges AND virtual vertices (Table 2 P:1566-1588:
+ * "GraphChi-vEN CC has both virtual edges and nodes"; readings
+ * G32/G33 in DESIGN.md). Same CSR, degree-bucket vertex types, constructor
+ * argument { u32 vid, u32 deg } and work entries as VF_APP_GRAPH.
+ *
+ * VF_APP_EDGE objects: one per arc k = (u -> v) of the symmetric CSR, type 0
+ * Edge, or 1 HubEdge when the source u is a Hub (deg >= 256); constructor
+ * argument { u32 src, u32 dst }. Layout (32 B): { vTable*, u32 src, u32 dst,
+ * union { double f[2]; u32 u[2]; } val } — a double-buffered edge value
+ * (Jacobi: iteration with buffer b reads val[b], the next reads val[1-b]).
+ * out_edges_dev[k] = pointer of arc k (the vertex's own arcs, CSR order);
+ * in_edges_dev[k] = pointer of the reverse arc (col[k] -> v) of arc k, so the
+ * in-edges of v are visited in ascending source order, the oracle's order.
+ *
+ * Inside a vertex method every edge access is a virtual call on the edge
+ * object (ChiEdge::target / get_pr / get_label). Under VF_CUDA / VF_SHAREDOA
+ * it is the compiler's virtual call (vTable* load, vFunc* load, indirect
+ * CALL); under VF_COAL / VF_TYPEPTR the vertex body is devirtualised and so
+ * are its edge calls: the edge type comes from the edge pointer by `er.rule`
+ * (VF_COAL: the edge app's range table; VF_TYPEPTR: the pointer's tag),
+ * unresolvable pointers fall back to the embedded vTable* (matched against
+ * er.vptr_dev), and the lanes of a warp are grouped by edge type for a
+ * direct, inlined call. Pointers in the edge arrays must be tagged under
+ * VF_TYPEPTR (vf_alloc_typed_batch(tag = 1)). */
+typedef struct {
+  const uint64_t* start_dev;   /* VF_APP_EDGE range table rows (vf_range_table), device copies */
+  const uint64_t* end_dev;
+  const uint32_t* type_dev;
+  const uint64_t* vptr_dev;    /* vf_type_vptrs(VF_APP_EDGE): 2 entries                          */
+  uint32_t K;                  /* rows                                                           */
+  uint32_t P;                  /* smallest power of two >= K                                     */
+  uint32_t rule;               /* VF_COAL or VF_TYPEPTR (used only by the COAL/TP kernels)        */
+} vf_edge_resolver;
+
+enum {
+  VF_GRAPH_EN_BFS_EXPAND = 0, /* top-down: for each out-edge e of the entry's chunk, u =
+                                 e->target(); claim depth[u] = level+1 (atomicCAS) and
+                                 append u's entries to next_queue / next_chunk           */
+  VF_GRAPH_EN_CC_UPDATE = 1,  /* m = min(label_in[v], e->get_label(b) over the chunk's
+                                 in-edges); label_out[v] = m (multi-chunk: atomicMin, as
+                                 VF_GRAPH_CC_UPDATE); *changed = 1 if m < label_in[v]     */
+  VF_GRAPH_EN_PR_INIT = 2,    /* chunk 0 only: contrib[v] = deg ? rank_in[v]/deg : 0;
+                                 deg-0 vertices add rank_in[v] to *dangling_out           */
+  VF_GRAPH_EN_PR_GATHER = 3   /* s = sum of e->get_pr(b) over the chunk's in-edges (fp64);
+                                 multi-chunk combine as VF_GRAPH_PR_UPDATE; r =
+                                 (float)(base + d*(s + *dangling_in/Vd)); rank_out[v] = r,
+                                 contrib[v] = deg ? r/deg : 0, deg-0: *dangling_out += r */
+};
+enum {
+  VF_EDGE_PULL_PR = 0,    /* val.f[slot] = contrib[src]  (the edge stores its source's share) */
+  VF_EDGE_PULL_LABEL = 1, /* val.u[slot] = label[src]                                         */
+  VF_EDGE_GET = 2         /* out[k] = (u64)src << 32 | dst, k = the entry index (verification) */
+};
+typedef struct {
+  const uint64_t* offs_dev;
+  const uint64_t* out_edges_dev;
+  int32_t* depth_dev;
+  const uint64_t* vobj_dev;
+  const uint32_t* chunk_dev;
+  uint64_t* next_queue_dev;
+  uint32_t* next_chunk_dev;
+  uint32_t* next_count_dev;
+  int32_t level;
+  uint32_t C;
+  vf_edge_resolver er;
+} vf_graph_en_bfs_args;
+typedef struct {
+  const uint64_t* offs_dev;
+  const uint64_t* in_edges_dev;
+  const uint32_t* label_in_dev;
+  uint32_t* label_out_dev;
+  uint32_t* changed_dev;
+  const uint32_t* chunk_dev;
+  uint32_t C;
+  uint32_t b;                  /* edge buffer read this iteration (0 / 1)                        */
+  vf_edge_resolver er;
+} vf_graph_en_cc_args;
+typedef struct {
+  const uint64_t* offs_dev;
+  const uint64_t* in_edges_dev;
+  const float* rank_in_dev;
+  float* rank_out_dev;
+  double* contrib_dev;
+  const double* dangling_in_dev;  /* D_t (read)                                                 */
+  double* dangling_out_dev;       /* D_{t+1} (accumulated; zeroed by the caller)                 */
+  double base, d, Vd;
+  const uint32_t* chunk_dev;
+  double* partial_dev;
+  uint32_t* counter_dev;
+  uint32_t C;
+  uint32_t b;
+  vf_edge_resolver er;
+} vf_graph_en_pr_args;
+typedef struct {
+  const double* contrib_dev;
+  const uint32_t* label_dev;
+  uint64_t* out_dev;           /* VF_EDGE_GET                                                    */
+  uint32_t slot;
+} vf_edge_args;
 
 #define VF_MAX_RANGES 4096u     /* COAL range-table capacity (staged in shared memory)   */
 #define VF_MAX_ARGS_BYTES 256u  /* method argument blob, copied into kernel parameters   */

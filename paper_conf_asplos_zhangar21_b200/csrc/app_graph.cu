@@ -11,7 +11,7 @@
 // 1.2-1.5x SLOWER than these per-lane loops at RMAT-24.)
 //
 // Object layout (16 B): { vTable* (8 B), u32 vid, u32 deg }.
-#include "dispatch.cuh"
+#include "graph_common.cuh"
 
 namespace vf {
 namespace graph {
@@ -34,67 +34,6 @@ struct Vertex {
   uint32_t vid;
   uint32_t deg;
 };
-
-// Neighbour loop with U independent lanes of work (U = 1: plain loop).
-template <int U, class F>
-__device__ __forceinline__ void for_neighbors(const uint32_t* __restrict__ col, uint64_t b, uint64_t e, F&& f) {
-  uint64_t k = b;
-  if constexpr (U > 1) {
-    for (; k + U <= e; k += U) {
-      uint32_t u[U];
-#pragma unroll
-      for (int j = 0; j < U; ++j) u[j] = __ldg(col + k + j);
-#pragma unroll
-      for (int j = 0; j < U; ++j) f(u[j]);
-    }
-  }
-  for (; k < e; ++k) f(__ldg(col + k));
-}
-
-__device__ __forceinline__ uint32_t nchunks(uint32_t deg, uint32_t C) { return deg <= C ? 1u : (deg + C - 1) / C; }
-
-// The edge range of work entry i of vertex (vid, deg): chunk c of <= C edges.
-// Single-chunk vertices (deg <= C, nearly all) never read the chunk array.
-struct Work {
-  uint64_t b, e;
-  uint32_t c, nch;
-};
-__device__ __forceinline__ Work work_of(const uint64_t* offs, const uint32_t* chunk, uint64_t i, uint32_t vid,
-                                        uint32_t deg, uint32_t C) {
-  Work w;
-  w.nch = nchunks(deg, C);
-  w.c = w.nch > 1 ? __ldg(chunk + i) : 0u;
-  const uint64_t b0 = __ldg(offs + vid);
-  w.b = b0 + (uint64_t)w.c * C;
-  const uint64_t e0 = b0 + deg;
-  w.e = w.b + C < e0 ? w.b + C : e0;
-  return w;
-}
-
-// Append vertex u's work entries to the next BFS frontier. Single-chunk
-// vertices reserve their slots with one warp-aggregated atomic per group of
-// lanes that claim at the same time, multi-chunk ones alone.
-__device__ __forceinline__ void enqueue(const vf_graph_bfs_args& a, uint32_t u) {
-  const uint32_t d = (uint32_t)(__ldg(a.offs_dev + u + 1) - __ldg(a.offs_dev + u));
-  const uint32_t n = nchunks(d, a.C);
-  const uint64_t obj = __ldg(a.vobj_dev + u);
-  if (n == 1) {
-    const uint32_t m = __activemask();
-    const uint32_t lane = threadIdx.x & 31u;
-    const uint32_t leader = __ffs(m) - 1;
-    uint32_t base = 0;
-    if (lane == leader) base = atomicAdd(a.next_count_dev, (uint32_t)__popc(m));
-    base = __shfl_sync(m, base, leader) + __popc(m & ((1u << lane) - 1u));
-    a.next_queue_dev[base] = obj;
-    a.next_chunk_dev[base] = 0;
-  } else {
-    const uint32_t base = atomicAdd(a.next_count_dev, n);
-    for (uint32_t j = 0; j < n; ++j) {
-      a.next_queue_dev[base + j] = obj;
-      a.next_chunk_dev[base + j] = j;
-    }
-  }
-}
 
 template <int KIND>
 struct VertexK final : Vertex {

@@ -42,6 +42,8 @@ static const AppOps* app_ops(uint32_t app) {
     case VF_APP_NBODY: return app_nbody();
     case VF_APP_STUT: return app_stut();
     case VF_APP_COLLIDE: return app_collide();
+    case VF_APP_GRAPH_EN: return app_graph_en();
+    case VF_APP_EDGE: return app_edge();
   }
   return nullptr;
 }

@@ -56,6 +56,16 @@ __device__ __forceinline__ uint64_t ldg_u64(const uint64_t* p) {
   return v;
 }
 
+// Methods whose bodies are long and of varying length (App::kHeavyMask bit M).
+template <class A, class = void>
+struct HeavyMaskOf {
+  static constexpr uint32_t value = 0;
+};
+template <class A>
+struct HeavyMaskOf<A, std::void_t<decltype(A::kHeavyMask)>> {
+  static constexpr uint32_t value = A::kHeavyMask;
+};
+
 __host__ __device__ constexpr size_t table_smem_dev(uint32_t P) { return (size_t)P * (8 + 8 + 4); }
 
 __device__ __forceinline__ void prefetch_l1(uint64_t a) {
@@ -451,14 +461,33 @@ __global__ void __launch_bounds__(kBlock, MinBlocks<App>::value) k_dispatch_sort
   uint32_t sink = 0;
   uint32_t hint = 0;  // COAL: last range hit by this lane
 
-  for (uint64_t base = (uint64_t)blockIdx.x * TILE; base < n; base += (uint64_t)gridDim.x * TILE) {
+  // Light methods keep the NEXT tile's pointers in flight (registers) while
+  // this tile is resolved, sorted and called: the pointer stream never waits
+  // for the tile's barriers.
+  constexpr bool kAhead = ((HeavyMaskOf<App>::value >> M) & 1u) == 0;
+  const uint64_t stride = (uint64_t)gridDim.x * TILE;
+  uint64_t pn[U];
+  if constexpr (kAhead) {
+#pragma unroll
+    for (int j = 0; j < U; ++j) {
+      const uint64_t idx = (uint64_t)blockIdx.x * TILE + (uint64_t)j * kBlock + threadIdx.x;
+      pn[j] = idx < n ? ldg_u64(objs + idx) : 0ull;
+    }
+  }
+  for (uint64_t base = (uint64_t)blockIdx.x * TILE; base < n; base += stride) {
     // A: pointers -> (type, address); warm the object lines
     uint64_t p[U], a[U];
     uint32_t t[U], w[U], rank[U];
 #pragma unroll
     for (int j = 0; j < U; ++j) {
-      const uint64_t idx = base + (uint64_t)j * kBlock + threadIdx.x;
-      p[j] = idx < n ? ldg_u64(objs + idx) : 0ull;
+      if constexpr (kAhead) {
+        p[j] = pn[j];
+        const uint64_t idx = base + stride + (uint64_t)j * kBlock + threadIdx.x;
+        pn[j] = idx < n ? ldg_u64(objs + idx) : 0ull;
+      } else {
+        const uint64_t idx = base + (uint64_t)j * kBlock + threadIdx.x;
+        p[j] = idx < n ? ldg_u64(objs + idx) : 0ull;
+      }
     }
 #pragma unroll
     for (int j = 0; j < U; ++j) {
@@ -484,6 +513,18 @@ __global__ void __launch_bounds__(kBlock, MinBlocks<App>::value) k_dispatch_sort
       mixed |= (pres & (pres - 1)) != 0;
     }
     const bool sorted = __syncthreads_or(mixed) != 0;  // CTA-uniform
+    if constexpr (((HeavyMaskOf<App>::value >> M) & 1u) == 0) {
+      // light bodies: a separate call site for type-uniform tiles (no selects
+      // on the sorted path, measured faster for config 2)
+      if (!sorted) {
+#pragma unroll
+        for (int j = 0; j < U; ++j) {
+          sink ^= w[j];
+          group_call<App, M>(t[j], a[j], 0ull, base + (uint64_t)j * kBlock + threadIdx.x, args, tbl);
+        }
+        continue;
+      }
+    }
     if (sorted) {
       // B: rank within type (warp-aggregated smem atomics)
 #pragma unroll
@@ -887,10 +928,28 @@ cudaError_t launch_grouped_pf(int pf, const uint64_t* objs, uint64_t n, const Ar
   return launch_grouped<App, M, R, U, 2>(objs, n, args, tbl, s);
 }
 
+// Apps with long bodies may set kLean: only the app's default grouped
+// configuration is instantiated (sorted tiles or, with regroup = 0, the plain
+// grouped kernel, each at kUnrollSorted / kUnroll and kPrefetch); the
+// unroll / prefetch / pipeline knobs do not apply. Keeps compile time bounded.
+template <class A, class = void>
+struct Lean {
+  static constexpr bool value = false;
+};
+template <class A>
+struct Lean<A, std::void_t<decltype(A::kLean)>> {
+  static constexpr bool value = A::kLean;
+};
+
 template <class App, int M, class R>
 cudaError_t launch_grouped_tuned(const uint64_t* objs, uint64_t n, const ArgBlob& args,
                                  const DevTable& tbl, cudaStream_t s) {
   const Tuning& tu = tuning();
+  if constexpr (Lean<App>::value) {
+    if (App::kTypes > 1 && tu.regroup != 0)
+      return launch_sorted<App, M, R, App::kUnrollSorted, App::kPrefetch>(objs, n, args, tbl, s);
+    return launch_grouped<App, M, R, App::kUnroll, App::kPrefetch>(objs, n, args, tbl, s);
+  } else {
   // Measured on B200 (config 2, 2^26 objects): with the per-tile type sort,
   // 2 objects per thread + L1 warm-up is best up to ~16 live types; with >= 24
   // live types (the sort leaves ~half-warp groups) 4 objects per thread
@@ -902,6 +961,7 @@ cudaError_t launch_grouped_tuned(const uint64_t* objs, uint64_t n, const ArgBlob
   if (u >= 4) return launch_grouped_pf<App, M, R, 4>(pf, objs, n, args, tbl, s);
   if (u == 2) return launch_grouped_pf<App, M, R, 2>(pf, objs, n, args, tbl, s);
   return launch_grouped_pf<App, M, R, 1>(pf, objs, n, args, tbl, s);
+  }
 }
 
 template <class App, int M, class R>

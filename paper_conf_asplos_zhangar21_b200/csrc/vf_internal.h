@@ -66,6 +66,8 @@ const AppOps* app_traf();
 const AppOps* app_nbody();
 const AppOps* app_stut();
 const AppOps* app_collide();
+const AppOps* app_graph_en();
+const AppOps* app_edge();
 
 // config 3 renderer (app_ray.cu): rows [row0, row0+nrows) of a W x H image
 cudaError_t ray_render(int variant, const uint64_t* objs, uint32_t S, uint32_t W, uint32_t H, uint32_t row0,

@@ -167,6 +167,44 @@ class gen_next_args(ctypes.Structure):
 gen_get_args = gol_get_args
 
 
+APP_GRAPH_EN, APP_EDGE = 9, 10
+GRAPH_EN_BFS_EXPAND, GRAPH_EN_CC_UPDATE, GRAPH_EN_PR_INIT, GRAPH_EN_PR_GATHER = 0, 1, 2, 3
+EDGE_PULL_PR, EDGE_PULL_LABEL, EDGE_GET = 0, 1, 2
+
+
+class edge_resolver(ctypes.Structure):
+    _fields_ = [("start_dev", ctypes.c_void_p), ("end_dev", ctypes.c_void_p), ("type_dev", ctypes.c_void_p),
+                ("vptr_dev", ctypes.c_void_p), ("K", ctypes.c_uint32), ("P", ctypes.c_uint32),
+                ("rule", ctypes.c_uint32)]
+
+
+class graph_en_bfs_args(ctypes.Structure):
+    _fields_ = [("offs_dev", ctypes.c_void_p), ("out_edges_dev", ctypes.c_void_p), ("depth_dev", ctypes.c_void_p),
+                ("vobj_dev", ctypes.c_void_p), ("chunk_dev", ctypes.c_void_p), ("next_queue_dev", ctypes.c_void_p),
+                ("next_chunk_dev", ctypes.c_void_p), ("next_count_dev", ctypes.c_void_p), ("level", ctypes.c_int32),
+                ("C", ctypes.c_uint32), ("er", edge_resolver)]
+
+
+class graph_en_cc_args(ctypes.Structure):
+    _fields_ = [("offs_dev", ctypes.c_void_p), ("in_edges_dev", ctypes.c_void_p), ("label_in_dev", ctypes.c_void_p),
+                ("label_out_dev", ctypes.c_void_p), ("changed_dev", ctypes.c_void_p), ("chunk_dev", ctypes.c_void_p),
+                ("C", ctypes.c_uint32), ("b", ctypes.c_uint32), ("er", edge_resolver)]
+
+
+class graph_en_pr_args(ctypes.Structure):
+    _fields_ = [("offs_dev", ctypes.c_void_p), ("in_edges_dev", ctypes.c_void_p), ("rank_in_dev", ctypes.c_void_p),
+                ("rank_out_dev", ctypes.c_void_p), ("contrib_dev", ctypes.c_void_p),
+                ("dangling_in_dev", ctypes.c_void_p), ("dangling_out_dev", ctypes.c_void_p),
+                ("base", ctypes.c_double), ("d", ctypes.c_double), ("Vd", ctypes.c_double),
+                ("chunk_dev", ctypes.c_void_p), ("partial_dev", ctypes.c_void_p), ("counter_dev", ctypes.c_void_p),
+                ("C", ctypes.c_uint32), ("b", ctypes.c_uint32), ("er", edge_resolver)]
+
+
+class edge_args(ctypes.Structure):
+    _fields_ = [("contrib_dev", ctypes.c_void_p), ("label_dev", ctypes.c_void_p), ("out_dev", ctypes.c_void_p),
+                ("slot", ctypes.c_uint32)]
+
+
 class graph_bfs_args(ctypes.Structure):
     _fields_ = [("offs_dev", ctypes.c_void_p), ("col_dev", ctypes.c_void_p), ("depth_dev", ctypes.c_void_p),
                 ("vobj_dev", ctypes.c_void_p), ("chunk_dev", ctypes.c_void_p), ("next_queue_dev", ctypes.c_void_p),

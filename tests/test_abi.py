@@ -95,3 +95,36 @@ def test_header_is_plain_c():
         r = subprocess.run(["gcc", "-fsyntax-only", "-x", lang, std, "-Wall", "-Werror", HDR],
                            capture_output=True, text=True)
         assert r.returncode == 0, r.stderr
+
+
+def test_arg_struct_layouts_match_header(tmp_path):
+    """The ctypes mirrors of the method-argument structs have the C sizes and
+    field offsets of include/vf.h (compiled here with gcc)."""
+    import ctypes
+    structs = {"vf_graph_en_bfs_args": vf.graph_en_bfs_args, "vf_graph_en_cc_args": vf.graph_en_cc_args,
+               "vf_graph_en_pr_args": vf.graph_en_pr_args, "vf_edge_args": vf.edge_args,
+               "vf_edge_resolver": vf.edge_resolver, "vf_graph_bfs_args": vf.graph_bfs_args,
+               "vf_graph_cc_args": vf.graph_cc_args, "vf_graph_pr_args": vf.graph_pr_args}
+    lines = ['#include <stdio.h>', '#include <stddef.h>', f'#include "{HDR}"', "int main(void) {"]
+    for cname, py in structs.items():
+        lines.append(f'  printf("{cname} %zu\\n", sizeof({cname}));')
+        for fname, _ in py._fields_:
+            lines.append(f'  printf("{cname}.{fname} %zu\\n", offsetof({cname}, {fname}));')
+    lines.append("  return 0;\n}")
+    src = tmp_path / "layout.c"
+    src.write_text("\n".join(lines))
+    exe = tmp_path / "layout"
+    subprocess.run(["gcc", "-std=c11", "-o", str(exe), str(src)], check=True)
+    got = dict(l.split() for l in subprocess.run([str(exe)], capture_output=True, text=True,
+                                                  check=True).stdout.splitlines())
+    for cname, py in structs.items():
+        assert int(got[cname]) == ctypes.sizeof(py), cname
+        for fname, _ in py._fields_:
+            assert int(got[f"{cname}.{fname}"]) == getattr(py, fname).offset, f"{cname}.{fname}"
+
+
+def test_graph_en_app_info():
+    nt, sizes, nm = vf.app_info(vf.APP_GRAPH_EN)
+    assert nt == 4 and nm == 4 and sizes == [16, 16, 16, 16]
+    nt, sizes, nm = vf.app_info(vf.APP_EDGE)
+    assert nt == 2 and nm == 3 and sizes == [32, 32]

@@ -27,6 +27,7 @@ import oracle  # noqa: E402  (cpu_baseline leg only)
 import synth  # noqa: E402
 from paper_conf_asplos_zhangar21_b200 import apps, vf  # noqa: E402
 from paper_conf_asplos_zhangar21_b200.graph import Graph  # noqa: E402
+from paper_conf_asplos_zhangar21_b200.graph_en import GraphEN  # noqa: E402
 from paper_conf_asplos_zhangar21_b200.ray import Ray  # noqa: E402
 from paper_conf_asplos_zhangar21_b200.traf import Traf  # noqa: E402
 from paper_conf_asplos_zhangar21_b200.nbody import Nbody  # noqa: E402
@@ -162,6 +163,57 @@ def bench_graph(ctx, quick):
         ctx.reset()
 
 
+# ---------------------------------------------------------------- §8f f4: GraphChi-vEN
+def _graph_en_scale(ctx, scale, variants, tag):
+    t0 = time.time()
+    offs, col = synth.rmat_graph(scale, seed=1)
+    V, A = len(offs) - 1, len(col)
+    print(f"# vEN rmat-{scale}: V={V} arcs={A} gen {time.time() - t0:.1f}s", flush=True)
+    types = synth.vertex_types(offs)
+    src = int(np.argmax(np.diff(offs.astype(np.int64))))
+    deg = np.diff(offs.astype(np.int64))
+    cpu = None
+    if scale <= 20:
+        _, _, bvc, bec, bsec = oracle.graph_en_bfs(offs, col, types, src)
+        _, it, cvc, cec, csec = oracle.graph_en_cc(offs, col, types)
+        _, psec = oracle.graph_en_pr(offs, col, types, iters=5)
+        cpu = dict(bfs=cpu_info(bvc + bec, bsec, f"rmat-{scale}, 1 thread"),
+                   cc=cpu_info(cvc + cec, csec, f"rmat-{scale}, 1 thread"),
+                   pr=cpu_info(5 * (V + 2 * A), psec, f"rmat-{scale}, 5 iterations, 1 thread"))
+    for v in variants:
+        g = GraphEN(ctx, offs, col, v)
+        ms = ev_time(lambda: g.bfs(src), 3, warm=1)
+        ec = g.edge_calls_bfs()
+        calls = g.vcalls + ec
+        # frontier entry: 8 ptr + 16 vertex + 8 offs; out-edge: 8 ptr + 4 dst + 4 depth
+        byts = 32 * g.vcalls + 16 * ec
+        record("graph-en-bfs", f"{tag} rmat-{scale} vEN top-down BFS", v, calls, ms, byts / calls, "GB/s", "hbm",
+               dict(V=V, arcs=A, vertex_calls=g.vcalls, edge_calls=ec), cpu and cpu["bfs"])
+        g.cc_init()
+        ms = ev_time(lambda: (g.changed.zero_(), g.cc_iteration()), 5, warm=2)
+        # vertex 8 ptr + 16 obj + 8 offs + 4 in + 4 out; in-edge get 8 ptr + 4; pull 8 ptr + 4 src + 4 lab + 4
+        calls = g.E + 2 * A
+        byts = 40 * g.E + 12 * A + 20 * A
+        record("graph-en-cc", f"{tag} rmat-{scale} vEN CC iteration", v, calls, ms, byts / calls, "GB/s", "hbm",
+               dict(vertex_calls=g.E, edge_calls=2 * A), cpu and cpu["cc"])
+        g.pr_init()
+        ms = ev_time(lambda: g.pr_iteration(), 5, warm=2)
+        # vertex 8 ptr + 16 obj + 8 offs + 4 rank + 8 contrib; in-edge get 8 ptr + 8; pull 8 ptr + 4 src + 8 + 8
+        byts = 44 * g.E + 16 * A + 28 * A
+        record("graph-en-pr", f"{tag} rmat-{scale} vEN PageRank iteration", v, calls, ms, byts / calls, "GB/s",
+               "hbm", dict(vertex_calls=g.E, edge_calls=2 * A), cpu and cpu["pr"])
+        del g
+        ctx.reset()
+        torch.cuda.empty_cache()
+
+
+def bench_graph_en(ctx, quick):
+    # the device-heap CUDA baseline allocates one `new` per edge (~3 us each): all
+    # four variants at rmat-18; the typed variants also at the config-4 scale
+    _graph_en_scale(ctx, 16 if quick else 18, VARIANTS, "all-variants")
+    _graph_en_scale(ctx, 20 if quick else 24, ("sharedoa", "coal", "typeptr"), "full")
+
+
 # ---------------------------------------------------------------- config 3: ray
 def bench_ray(ctx, quick):
     W, H, S = (480, 270, 10000) if quick else (1920, 1080, 10000)
@@ -286,7 +338,8 @@ def main():
         f.write("| app | config | variant | calls/step | ms/step | Gcalls/s | vs cuda | achieved | frac | "
                 "oracle Gcalls/s (cores) |\n|---|---|---|---|---|---|---|---|---|---|\n")
         for r in ROWS:
-            base = next((x for x in ROWS if x["app"] == r["app"] and x["variant"] == "cuda"), None)
+            base = next((x for x in ROWS if x["app"] == r["app"] and x["config"] == r["config"]
+                         and x["variant"] == "cuda"), None)
             rel = r["calls_per_s"] / base["calls_per_s"] if base else float("nan")
             rf = r["roofline"]
             cpu = r.get("cpu_baseline")

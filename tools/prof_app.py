@@ -28,7 +28,20 @@ def main():
     ap.add_argument("--steps", type=int, default=3)
     a = ap.parse_args()
     ctx = vf.Ctx(0, cuda_heap_bytes=8 << 30)
-    if a.app.startswith("graph"):
+    if a.app.startswith("graph-en"):
+        from paper_conf_asplos_zhangar21_b200.graph_en import GraphEN
+        offs, col = synth.rmat_graph(a.scale, seed=1)
+        g = GraphEN(ctx, offs, col, a.variant)
+        src = int(np.argmax(np.diff(offs.astype(np.int64))))
+        if a.app == "graph-en-pr":
+            g.pr_init()
+            for _ in range(a.steps):
+                g.pr_iteration()
+        elif a.app == "graph-en-cc":
+            g.cc(max_iters=a.steps)
+        else:
+            g.bfs(src)
+    elif a.app.startswith("graph"):
         from paper_conf_asplos_zhangar21_b200.graph import Graph
         offs, col = synth.rmat_graph(a.scale, seed=1)
         g = Graph(ctx, offs, col, a.variant)
