@@ -557,6 +557,17 @@ vf_status vf_gen_swap(vf_ctx* ctx, uint64_t ncells, const uint8_t* state_prev_de
 vf_status vf_gol_step(vf_ctx* ctx, vf_variant v, uint32_t W, uint32_t H, int torus, const uint8_t* state_prev_dev,
                       uint8_t* state_next_dev, uint8_t* nbr_dev, uint64_t* grid_dev, const uint64_t* alive_dev,
                       const uint64_t* dead_dev, void* stream);
+/* `gens` generations of vf_gol_step in ONE cooperative launch (config 1 is
+ * launch-latency bound: a 256 x 256 generation is a few microseconds of
+ * work). Generation g reads state[g & 1] and writes state[(g + 1) & 1]
+ * (state0 = the current state; after the call the current state is
+ * state[gens & 1]); generations are separated by a grid barrier on
+ * *barrier_dev (caller-owned u32, zeroed by the call on `stream`). Every
+ * variant runs the same structure; results are identical to `gens` calls of
+ * vf_gol_step. VF_ERR_CUDA if the grid cannot be co-resident. */
+vf_status vf_gol_run(vf_ctx* ctx, vf_variant v, uint32_t W, uint32_t H, int torus, uint8_t* state0_dev,
+                     uint8_t* state1_dev, uint8_t* nbr_dev, uint64_t* grid_dev, const uint64_t* alive_dev,
+                     const uint64_t* dead_dev, uint32_t gens, uint32_t* barrier_dev, void* stream);
 /* Same for GEN (VF_GEN_NEXT with {nbr, next, born_mask, survive_mask, C}, then vf_gen_swap). */
 vf_status vf_gen_step(vf_ctx* ctx, vf_variant v, uint32_t W, uint32_t H, int torus, const uint8_t* state_prev_dev,
                       uint8_t* state_next_dev, uint8_t* nbr_dev, uint64_t* grid_dev, const uint64_t* dead_dev,

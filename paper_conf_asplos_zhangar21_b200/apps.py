@@ -130,6 +130,16 @@ class Gol:
             vf.gol_swap(self.ctx, cur, nxt, self.grid, self.alive, self.dead, stream)
         self.parity ^= 1
 
+    def run(self, gens: int, stream=None):
+        """`gens` generations in ONE persistent cooperative launch (vf_gol_run):
+        same results as `gens` calls of gen()."""
+        if not hasattr(self, "barrier"):
+            self.barrier = torch.zeros(1, dtype=torch.int32, device=self.grid.device)
+        s0, s1 = (self.state, self.next) if self.parity == 0 else (self.next, self.state)
+        vf.gol_run(self.ctx, self.v, self.W, self.H, self.torus, s0, s1, self.nbr, self.grid, self.alive, self.dead,
+                   gens, self.barrier, stream)
+        self.parity ^= gens & 1
+
     @property
     def current(self):
         return self.state if self.parity == 0 else self.next

@@ -126,6 +126,141 @@ struct Step {
   }
 };
 
+
+// ---------------------------------------------------------------------------
+// Persistent multi-generation run (vf_gol_run). At 256 x 256 one generation is
+// a few microseconds of work, so a launch per generation is launch-latency
+// bound. Here ONE cooperative launch runs all generations: every cell is
+// owned by a fixed thread (grid-stride mapping with a fixed grid), generations
+// are separated by a grid barrier, and COAL's range table is staged into
+// shared memory once for all of them. State arrays written by other CTAs are
+// read with ld.global.cg (L2; L1 is not coherent across SMs); everything else
+// a thread touches (its cells' nbr, grid entries and objects) is its own.
+// Same variants, same bodies, same results as vf_gol_step per generation.
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ uint8_t ldcg_u8(const uint8_t* p) { return __ldcg(p); }
+
+__device__ __forceinline__ uint8_t count_live_cg(uint32_t W, uint32_t H, int torus, const uint8_t* st, uint64_t c) {
+  const int y = (int)(c / W), x = (int)(c % W);
+  int n = 0;
+#pragma unroll
+  for (int dy = -1; dy <= 1; ++dy)
+#pragma unroll
+    for (int dx = -1; dx <= 1; ++dx) {
+      if (dx == 0 && dy == 0) continue;
+      int yy = y + dy, xx = x + dx;
+      if (torus) {
+        yy = (yy + (int)H) % (int)H;
+        xx = (xx + (int)W) % (int)W;
+      } else if (yy < 0 || yy >= (int)H || xx < 0 || xx >= (int)W) {
+        continue;
+      }
+      n += ldcg_u8(st + (uint64_t)yy * W + xx) == 1;
+    }
+  return (uint8_t)n;
+}
+
+__device__ __forceinline__ uint32_t ld_acquire_u32(const unsigned* p) {
+  uint32_t v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+
+// Monotonic grid barrier: after the g-th barrier *ctr == g * gridDim.x
+// (zeroed before the launch; all CTAs are co-resident: cooperative launch).
+__device__ __forceinline__ void grid_barrier(unsigned* ctr, uint32_t& target) {
+  __syncthreads();
+  target += gridDim.x;
+  if (threadIdx.x == 0) {
+    __threadfence();
+    atomicAdd(ctr, 1u);
+    while (ld_acquire_u32(ctr) < target) {
+    }
+  }
+  __syncthreads();
+}
+
+struct RunArgs {
+  uint32_t W, H;
+  int torus;
+  uint32_t gens;
+  uint8_t* buf[2];  // state buffers: generation g reads buf[g & 1], writes buf[(g + 1) & 1]
+  uint8_t* nbr;
+  uint64_t* grid;
+  const uint64_t* alive;
+  const uint64_t* dead;
+  unsigned* bar;
+};
+
+__device__ __forceinline__ void post_cg(const RunArgs& r, const uint8_t* prev, const uint8_t* next, uint64_t c) {
+  const uint8_t s = __ldcg(next + c);
+  if (s != __ldcg(prev + c)) {
+    const uint64_t p = s ? r.alive[c] : r.dead[c];
+    r.grid[c] = p;
+    reinterpret_cast<Cell*>(strip(p))->counter = 0;
+  }
+}
+
+template <class R>
+__global__ void __launch_bounds__(kBlock) k_run_grouped(RunArgs r, DevTable tbl) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  if constexpr (R::kNeedsTable) R::stage(smem, tbl);
+  const uint64_t n = (uint64_t)r.W * r.H;
+  uint32_t hint = 0, target = 0;
+  for (uint32_t g = 0; g < r.gens; ++g) {
+    const uint8_t* prev = r.buf[g & 1];
+    uint8_t* next = r.buf[(g + 1) & 1];
+    ArgBlob args{};
+    const vf_gol_next_args a{r.nbr, next};
+    *reinterpret_cast<vf_gol_next_args*>(args.b) = a;
+    for (uint64_t base = (uint64_t)blockIdx.x * kBlock; base < n; base += (uint64_t)gridDim.x * kBlock) {
+      const uint64_t c = base + threadIdx.x;
+      const bool valid = c < n;
+      uint64_t p = 0, ad = 0;
+      uint32_t t = kNF;
+      if (valid) {
+        r.nbr[c] = count_live_cg(r.W, r.H, r.torus, prev, c);
+        p = r.grid[c];
+      }
+      if (p) t = R::resolve(smem, tbl.P, p, ad, hint);
+      group_call<App, VF_GOL_NEXT>(t, ad, p, c, args, tbl);
+      if (valid) post_cg(r, prev, next, c);
+    }
+    grid_barrier(r.bar, target);
+  }
+}
+
+__global__ void __launch_bounds__(kBlock) k_run_virtual(RunArgs r) {
+  const uint64_t n = (uint64_t)r.W * r.H;
+  uint32_t target = 0;
+  for (uint32_t g = 0; g < r.gens; ++g) {
+    const uint8_t* prev = r.buf[g & 1];
+    uint8_t* next = r.buf[(g + 1) & 1];
+    const vf_gol_next_args a{r.nbr, next};
+    for (uint64_t c = (uint64_t)blockIdx.x * kBlock + threadIdx.x; c < n; c += (uint64_t)gridDim.x * kBlock) {
+      r.nbr[c] = count_live_cg(r.W, r.H, r.torus, prev, c);
+      const uint64_t p = r.grid[c];
+      if (p) reinterpret_cast<Cell*>(p)->next(a);  // the compiler's virtual call
+      post_cg(r, prev, next, c);
+    }
+    grid_barrier(r.bar, target);
+  }
+}
+
+template <class K>
+static cudaError_t coop_launch(K kern, uint64_t n, size_t sm, void** params, cudaStream_t s) {
+  int occ = 0;
+  if (sm > 48 * 1024) cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+  cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kBlock, sm);
+  if (e != cudaSuccess) return e;
+  if (occ < 1) return cudaErrorCooperativeLaunchTooLarge;
+  const uint64_t tiles = (n + kBlock - 1) / kBlock;
+  const uint64_t cap = (uint64_t)num_sms() * occ;
+  const unsigned grid = (unsigned)(tiles < cap ? (tiles ? tiles : 1) : cap);
+  e = cudaLaunchCooperativeKernel((const void*)kern, dim3(grid), dim3(kBlock), params, sm, s);
+  note_launch();
+  return e;
+}
 }  // namespace gol
 
 cudaError_t gol_step(int variant, uint32_t W, uint32_t H, int torus, const uint8_t* prev, uint8_t* next, uint8_t* nbr,
@@ -136,6 +271,28 @@ cudaError_t gol_step(int variant, uint32_t W, uint32_t H, int torus, const uint8
   memcpy(blob.b, &a, sizeof a);
   const gol::Step st{W, H, torus, prev, next, nbr, grid, alive, dead};
   return launch_step<gol::App, VF_GOL_NEXT>(variant, (uint64_t)W * H, blob, tbl, st, s);
+}
+
+cudaError_t gol_run(int variant, uint32_t W, uint32_t H, int torus, uint8_t* buf0, uint8_t* buf1, uint8_t* nbr,
+                    uint64_t* grid, const uint64_t* alive, const uint64_t* dead, uint32_t gens, unsigned* bar,
+                    const DevTable& tbl, cudaStream_t s) {
+  const uint64_t n = (uint64_t)W * H;
+  if (!gens || !n) return cudaSuccess;
+  cudaError_t e = cudaMemsetAsync(bar, 0, sizeof(unsigned), s);
+  if (e != cudaSuccess) return e;
+  gol::RunArgs r{W, H, torus, gens, {buf0, buf1}, nbr, grid, alive, dead, bar};
+  DevTable t = tbl;
+  void* params[2] = {&r, &t};
+  switch (variant) {
+    case VF_CUDA:
+    case VF_SHAREDOA:
+      return gol::coop_launch(gol::k_run_virtual, n, 0, params, s);
+    case VF_COAL:
+      return gol::coop_launch(gol::k_run_grouped<ResolveCOAL>, n, table_smem(tbl), params, s);
+    case VF_TYPEPTR:
+      return gol::coop_launch(gol::k_run_grouped<ResolveTP>, n, 0, params, s);
+  }
+  return cudaErrorInvalidValue;
 }
 
 static const uint32_t kGolBytes[2] = {16, 16};

@@ -110,22 +110,43 @@ __device__ __forceinline__ double e_get_pr(const EdgeK<K>* e, uint32_t b) { retu
 template <int K>
 __device__ __forceinline__ uint32_t e_get_label(const EdgeK<K>* e, uint32_t b) { return e->EdgeK<K>::get_label(b); }
 
-// Type of edge pointer p from its value (COAL range search over the edge
-// app's small table, L1-resident; or the TypePointer tag), else from the
-// embedded vTable*. a = the address to dereference.
-__device__ __forceinline__ uint32_t edge_type(const vf_edge_resolver& r, uint64_t p, uint64_t& a) {
+// COAL for edges: the two most recently hit ranges of the edge app's table are
+// kept in registers (an out-edge list is all one type; an in-edge list mixes
+// the two edge types), so the branch-free search over the table (L1-resident,
+// global memory) runs only on a miss.
+struct EdgeRangeCache {
+  uint64_t s0 = ~0ull, e0 = 0, s1 = ~0ull, e1 = 0;
+  uint32_t t0 = kNF, t1 = kNF;
+};
+
+// Type of edge pointer p from its value (COAL: cached ranges, else the range
+// search; TypePointer: the tag), else from the embedded vTable*. a = the
+// address to dereference.
+__device__ __forceinline__ uint32_t edge_type(const vf_edge_resolver& r, EdgeRangeCache& rc, uint64_t p,
+                                              uint64_t& a) {
   uint32_t t;
   if (r.rule == VF_TYPEPTR) {
     a = strip(p);
     t = ((uint32_t)(p >> 32) >> (VF_VA_BITS - 32)) - 1u;
   } else {
     a = p;
-    uint32_t j = 0;
-    for (uint32_t step = r.P >> 1; step > 0; step >>= 1) {
-      const uint32_t c = j + step;
-      j = (c < r.K && __ldg(r.start_dev + c) <= p) ? c : j;
+    if ((rc.s0 <= p) & (p < rc.e0)) {
+      t = rc.t0;
+    } else if ((rc.s1 <= p) & (p < rc.e1)) {
+      t = rc.t1;
+    } else {
+      uint32_t j = 0;
+      for (uint32_t step = r.P >> 1; step > 0; step >>= 1) {
+        const uint32_t c = j + step;
+        j = (c < r.K && __ldg(r.start_dev + c) <= p) ? c : j;
+      }
+      const uint64_t s = __ldg(r.start_dev + j), e = __ldg(r.end_dev + j);
+      t = (s <= p && p < e) ? __ldg(r.type_dev + j) : kNF;
+      if (t != kNF) {
+        rc.s1 = rc.s0, rc.e1 = rc.e0, rc.t1 = rc.t0;
+        rc.s0 = s, rc.e0 = e, rc.t0 = t;
+      }
     }
-    t = (__ldg(r.start_dev + j) <= p && p < __ldg(r.end_dev + j)) ? __ldg(r.type_dev + j) : kNF;
   }
   if (t >= (uint32_t)EdgeApp::kTypes) {  // fallback
     const uint64_t vp = *reinterpret_cast<const uint64_t*>(a);
@@ -138,13 +159,14 @@ __device__ __forceinline__ uint32_t edge_type(const vf_edge_resolver& r, uint64_
 // all, then run each edge type present among the active lanes' batches once,
 // over every slot of that type (independent loads stay in flight together).
 template <int U, class F>
-__device__ __forceinline__ void visit_direct(const vf_edge_resolver& r, const uint64_t (&p)[U], F&& f) {
+__device__ __forceinline__ void visit_direct(const vf_edge_resolver& r, EdgeRangeCache& rc, const uint64_t (&p)[U],
+                                             F&& f) {
   uint64_t a[U];
   uint32_t t[U];
   uint32_t mine = 0;
 #pragma unroll
   for (int j = 0; j < U; ++j) {
-    t[j] = edge_type(r, p[j], a[j]);
+    t[j] = edge_type(r, rc, p[j], a[j]);
     mine |= t[j] < (uint32_t)EdgeApp::kTypes ? 1u << t[j] : 0u;
   }
   const uint32_t present = __reduce_or_sync(__activemask(), mine);
@@ -161,31 +183,41 @@ __device__ __forceinline__ void visit_direct(const vf_edge_resolver& r, const ui
 }
 
 template <bool DIRECT, int U, class F>
-__device__ __forceinline__ void visit(const vf_edge_resolver& r, const uint64_t (&p)[U], F&& f) {
+__device__ __forceinline__ void visit(const vf_edge_resolver& r, EdgeRangeCache& rc, const uint64_t (&p)[U], F&& f) {
   if constexpr (DIRECT) {
-    visit_direct<U>(r, p, f);
+    visit_direct<U>(r, rc, p, f);
   } else {
 #pragma unroll
     for (int j = 0; j < U; ++j) f(j, reinterpret_cast<const ChiEdge*>(p[j]));
   }
 }
 
-// Edge k in [b, e) of a pointer array (out- or in-edges), U per batch.
-template <bool DIRECT, int U, class F>
+// Edge k in [b, e) of a pointer array (out- or in-edges), U per batch: the
+// edge call `get` (an accessor: target / get_label / get_pr) yields one value
+// per slot inside the type groups; `use(j, value)` then consumes the slots in
+// edge order outside them (one copy of the vertex's own logic, all lanes
+// converged, whatever mix of edge types the batch held).
+template <class T, bool DIRECT, int U, class G, class C>
 __device__ __forceinline__ void for_edges(const vf_edge_resolver& r, const uint64_t* __restrict__ ptrs, uint64_t b,
-                                          uint64_t e, F&& f) {
+                                          uint64_t e, G&& get, C&& use) {
+  EdgeRangeCache rc;
   uint64_t k = b;
   if constexpr (U > 1) {
     for (; k + U <= e; k += U) {
       uint64_t p[U];
 #pragma unroll
       for (int j = 0; j < U; ++j) p[j] = ldg_u64(ptrs + k + j);
-      visit<DIRECT, U>(r, p, f);
+      T v[U];
+      visit<DIRECT, U>(r, rc, p, [&](int j, auto* ed) { v[j] = get(ed); });
+#pragma unroll
+      for (int j = 0; j < U; ++j) use(j, v[j]);
     }
   }
   for (; k < e; ++k) {
     const uint64_t p[1] = {ldg_u64(ptrs + k)};
-    visit<DIRECT, 1>(r, p, f);
+    T v[1];
+    visit<DIRECT, 1>(r, rc, p, [&](int j, auto* ed) { v[j] = get(ed); });
+    use(0, v[0]);
   }
 }
 
@@ -217,16 +249,17 @@ __device__ __forceinline__ void add_dangling(double* D, float r) {
 
 template <int KIND>
 struct VertexK final : ChiVertex {
-  static constexpr int U = KIND <= 1 ? 1 : KIND == 2 ? 4 : 8;
+  static constexpr int U = KIND <= 1 ? 1 : 4;
   __device__ explicit VertexK(const void* arg) : ChiVertex(arg) {}
 
   template <bool D>
   __device__ __forceinline__ void bfs_expand_t(const vf_graph_en_bfs_args& a, uint64_t i) {
     const Work w = work_of(a.offs_dev, a.chunk_dev, i, vid, deg, a.C);
-    for_edges<D, U>(a.er, a.out_edges_dev, w.b, w.e, [&](int, auto* e) {
-      const uint32_t u = e_target(e);  // edge call
-      if (a.depth_dev[u] == -1 && atomicCAS(a.depth_dev + u, -1, a.level + 1) == -1) graph::enqueue(a, u);
-    });
+    for_edges<uint32_t, D, U>(
+        a.er, a.out_edges_dev, w.b, w.e, [](auto* e) { return e_target(e); },  // edge call
+        [&](int, uint32_t u) {
+          if (a.depth_dev[u] == -1 && atomicCAS(a.depth_dev + u, -1, a.level + 1) == -1) graph::enqueue(a, u);
+        });
   }
   template <bool D>
   __device__ __forceinline__ void cc_update_t(const vf_graph_en_cc_args& a, uint64_t i) {
@@ -235,8 +268,10 @@ struct VertexK final : ChiVertex {
     uint32_t acc[U];
 #pragma unroll
     for (int j = 0; j < U; ++j) acc[j] = own;
-    for_edges<D, U>(a.er, a.in_edges_dev, w.b, w.e,
-                    [&](int j, auto* e) { acc[j] = min(acc[j], e_get_label(e, a.b)); });  // edge call
+    const uint32_t b = a.b;
+    for_edges<uint32_t, D, U>(
+        a.er, a.in_edges_dev, w.b, w.e, [b](auto* e) { return e_get_label(e, b); },  // edge call
+        [&](int j, uint32_t x) { acc[j] = min(acc[j], x); });
     uint32_t m = own;
 #pragma unroll
     for (int j = 0; j < U; ++j) m = min(m, acc[j]);
@@ -256,8 +291,10 @@ struct VertexK final : ChiVertex {
     double acc[U];
 #pragma unroll
     for (int j = 0; j < U; ++j) acc[j] = 0.0;
-    for_edges<D, U>(a.er, a.in_edges_dev, w.b, w.e,
-                    [&](int j, auto* e) { acc[j] += e_get_pr(e, a.b); });  // edge call
+    const uint32_t b = a.b;
+    for_edges<double, D, U>(
+        a.er, a.in_edges_dev, w.b, w.e, [b](auto* e) { return e_get_pr(e, b); },  // edge call
+        [&](int j, double x) { acc[j] += x; });
     double s = 0.0;
 #pragma unroll
     for (int j = 0; j < U; ++j) s += acc[j];
@@ -295,6 +332,7 @@ struct VtxApp {
   static constexpr int kPrefetch = 2;
   static constexpr uint32_t kHeavyMask = 0xBu;  // bfs, cc, gather: one tile per CTA
   static constexpr bool kLean = true;           // default launch configuration only
+  static constexpr int kMinBlocks = 3;          // <= 80 registers: random edge gathers need warps
   using Base = ChiVertex;
   template <int K>
   using Type = VertexK<K>;

@@ -760,6 +760,23 @@ vf_status vf_gol_step(vf_ctx* c, vf_variant v, uint32_t W, uint32_t H, int torus
   return VF_OK;
 }
 
+vf_status vf_gol_run(vf_ctx* c, vf_variant v, uint32_t W, uint32_t H, int torus, uint8_t* state0_dev,
+                     uint8_t* state1_dev, uint8_t* nbr_dev, uint64_t* grid_dev, const uint64_t* alive_dev,
+                     const uint64_t* dead_dev, uint32_t gens, uint32_t* barrier_dev, void* stream) {
+  vf_status st = check_app(c, VF_APP_GOL);
+  if (st) return st;
+  if ((unsigned)v > VF_TYPEPTR) return fail(c, VF_ERR_INVALID, "variant %d", (int)v);
+  if ((uint64_t)W * H && gens &&
+      (!state0_dev || !state1_dev || !nbr_dev || !grid_dev || !alive_dev || !dead_dev || !barrier_dev))
+    return fail(c, VF_ERR_INVALID, "gol_run arguments");
+  if ((st = set_device(c)) || (st = ensure_vptrs(c, VF_APP_GOL))) return st;
+  if (v == VF_COAL && c->tables[VF_APP_GOL].K > VF_MAX_RANGES)
+    return fail(c, VF_ERR_TABLE_FULL, "K = %u > %u", c->tables[VF_APP_GOL].K, VF_MAX_RANGES);
+  CUDA_TRY(c, gol_run((int)v, W, H, torus, state0_dev, state1_dev, nbr_dev, grid_dev, alive_dev, dead_dev, gens,
+                      barrier_dev, dev_table(c, VF_APP_GOL), reinterpret_cast<cudaStream_t>(stream)));
+  return VF_OK;
+}
+
 vf_status vf_gen_step(vf_ctx* c, vf_variant v, uint32_t W, uint32_t H, int torus, const uint8_t* prev_dev,
                       uint8_t* next_dev, uint8_t* nbr_dev, uint64_t* grid_dev, const uint64_t* dead_dev,
                       const uint64_t* alive_dev, const uint64_t* dying_dev, uint32_t born_mask,

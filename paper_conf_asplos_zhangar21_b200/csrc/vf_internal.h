@@ -78,6 +78,9 @@ cudaError_t ray_render(int variant, const uint64_t* objs, uint32_t S, uint32_t W
 cudaError_t gol_step(int variant, uint32_t W, uint32_t H, int torus, const uint8_t* prev, uint8_t* next, uint8_t* nbr,
                      uint64_t* grid, const uint64_t* alive, const uint64_t* dead, const DevTable& tbl,
                      cudaStream_t s);
+cudaError_t gol_run(int variant, uint32_t W, uint32_t H, int torus, uint8_t* buf0, uint8_t* buf1, uint8_t* nbr,
+                    uint64_t* grid, const uint64_t* alive, const uint64_t* dead, uint32_t gens, unsigned* bar,
+                    const DevTable& tbl, cudaStream_t s);
 cudaError_t gen_step(int variant, uint32_t W, uint32_t H, int torus, const uint8_t* prev, uint8_t* next, uint8_t* nbr,
                      uint64_t* grid, const uint64_t* dead, const uint64_t* alive, const uint64_t* dying,
                      uint32_t born, uint32_t survive, uint32_t C, const DevTable& tbl, cudaStream_t s);

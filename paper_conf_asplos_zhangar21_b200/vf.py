@@ -39,7 +39,7 @@ SYMBOLS = [
     "vf_regions", "vf_type_vptrs", "vf_resolve", "vf_verify_types", "vf_dispatch_cuda",
     "vf_dispatch_sharedoa", "vf_dispatch_coal", "vf_dispatch_typeptr", "vf_dispatch",
     "vf_gol_neighbors", "vf_gol_swap", "vf_gen_swap", "vf_checksum_i32", "vf_launch_count", "vf_set_tuning",
-    "vf_graph_bfs_init", "vf_iota_u32", "vf_fill_f32", "vf_ray_render", "vf_gol_step", "vf_gen_step",
+    "vf_graph_bfs_init", "vf_iota_u32", "vf_fill_f32", "vf_ray_render", "vf_gol_step", "vf_gen_step", "vf_gol_run",
     "vf_dispatch_concord", "vf_micro_branch", "vf_collide_tmp_words", "vf_collide_grid",
 ]
 APP_RAY = 4
@@ -270,6 +270,7 @@ def lib(required: bool = True):
         "vf_fill_f32": (I, [U64, P, ctypes.c_float, P]),
         "vf_ray_render": (I, [P, I, P, U32, U32, U32, U32, U32, P, P, P, P, P]),
         "vf_gol_step": (I, [P, I, U32, U32, I, P, P, P, P, P, P, P]),
+        "vf_gol_run": (I, [P, I, U32, U32, I, P, P, P, P, P, P, U32, P, P]),
         "vf_dispatch_concord": (I, [P, U32, U32, P, U64, P, ctypes.c_size_t, P]),
         "vf_micro_branch": (I, [U64, U32, I, U64, U32, P, P]),
         "vf_collide_tmp_words": (U64, [U32, U32]),
@@ -472,6 +473,13 @@ def gol_step(ctx: Ctx, variant: int, W, H, torus, prev, nxt, nbr, grid, alive, d
                            _ptr(alive), _ptr(dead), _stream(stream))
     if st:
         ctx._check(st, "gol_step")
+
+
+def gol_run(ctx: Ctx, variant: int, W, H, torus, state0, state1, nbr, grid, alive, dead, gens, barrier, stream=None):
+    st = lib().vf_gol_run(ctx.h, variant, W, H, int(torus), _ptr(state0), _ptr(state1), _ptr(nbr), _ptr(grid),
+                          _ptr(alive), _ptr(dead), gens, _ptr(barrier), _stream(stream))
+    if st:
+        ctx._check(st, "gol_run")
 
 
 def gen_step(ctx: Ctx, variant: int, W, H, torus, prev, nxt, nbr, grid, dead, alive, dying, born, survive, C,

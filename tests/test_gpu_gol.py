@@ -67,3 +67,24 @@ def test_gol_cuda_graph_capture(ctx):
     graph.replay()
     torch.cuda.synchronize()
     assert np.array_equal(g.current.cpu().numpy(), st_ref)
+
+
+@pytest.mark.parametrize("variant", VARIANTS)
+@pytest.mark.parametrize("W,H,gens,torus", [(256, 256, 100, False), (37, 23, 31, False), (64, 48, 25, True),
+                                            (1024, 1024, 7, False)])
+def test_gol_persistent_run(ctx, variant, W, H, gens, torus):
+    """vf_gol_run: all generations in one cooperative launch (grid barrier between
+    generations; at 1024^2 each thread owns several cells) == the oracle."""
+    g0 = synth.soup(W, H, seed=43)
+    st_ref, ctr_ref, _, _ = oracle.gol_run(W, H, g0, gens, torus)
+    g = apps.Gol(ctx, W, H, g0, variant, torus)
+    g.run(gens)
+    assert np.array_equal(g.current.cpu().numpy(), st_ref)
+    ctr, typ = g.counters()
+    assert np.array_equal(ctr.cpu().numpy().view(np.uint16), ctr_ref)
+    assert np.array_equal(typ.cpu().numpy(), st_ref)
+    # split runs continue where the last one stopped
+    g2 = apps.Gol(ctx, W, H, g0, variant, torus)
+    g2.run(gens // 2)
+    g2.run(gens - gens // 2)
+    assert np.array_equal(g2.current.cpu().numpy(), st_ref)

@@ -96,7 +96,11 @@ def bench_gol(ctx, quick):
         # 8 B ptr + 1 B nbr + 1 B state out + 4 B counter r/w per next() call
         record("gol", "256x256, 100 gens (CUDA graph of 100 generations)", v, W * H, ms, 14, "GB/s", "l2/latency",
                dict(ms_per_gen_eager=ms_eager, ms_per_gen_eager_unfused=ms_unfused), cpu)
-        del g, graph
+        del graph
+        ms_run = ev_time(lambda: g.run(gens), 5) / gens
+        record("gol-run", "256x256, 100 gens in one persistent cooperative launch (vf_gol_run)", v, W * H, ms_run,
+               14, "GB/s", "l2/latency", None, cpu)
+        del g
     ctx.reset()
 
 
@@ -207,11 +211,15 @@ def _graph_en_scale(ctx, scale, variants, tag):
         torch.cuda.empty_cache()
 
 
+EN_FULL = True
+
+
 def bench_graph_en(ctx, quick):
     # the device-heap CUDA baseline allocates one `new` per edge (~3 us each): all
     # four variants at rmat-18; the typed variants also at the config-4 scale
     _graph_en_scale(ctx, 16 if quick else 18, VARIANTS, "all-variants")
-    _graph_en_scale(ctx, 20 if quick else 24, ("sharedoa", "coal", "typeptr"), "full")
+    if EN_FULL:
+        _graph_en_scale(ctx, 20 if quick else 24, ("sharedoa", "coal", "typeptr"), "full")
 
 
 # ---------------------------------------------------------------- config 3: ray
@@ -323,7 +331,10 @@ def main():
     ap.add_argument("--out", default="gpurun_out/apps")
     ap.add_argument("--quick", action="store_true")
     ap.add_argument("--tune", action="append", default=[], help="libvf tuning knob key=value (vf_set_tuning)")
+    ap.add_argument("--en-small-only", action="store_true", help="graph_en: rmat-18 (all variants) only")
     a = ap.parse_args()
+    global EN_FULL
+    EN_FULL = not a.en_small_only
     for kv in a.tune:
         k, v = kv.split("=")
         vf.set_tuning(k, int(v))
