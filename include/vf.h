@@ -562,7 +562,11 @@ vf_status vf_gol_step(vf_ctx* ctx, vf_variant v, uint32_t W, uint32_t H, int tor
  * work). Generation g reads state[g & 1] and writes state[(g + 1) & 1]
  * (state0 = the current state; after the call the current state is
  * state[gens & 1]); generations are separated by a grid barrier on
- * *barrier_dev (caller-owned u32, zeroed by the call on `stream`). Every
+ * *barrier_dev (caller-owned u32, zeroed by the call on `stream`), or, for
+ * grids of <= 2^17 cells, the launch is ONE thread-block cluster of up to 16
+ * CTAs that keeps the state rows in distributed shared memory and separates
+ * generations with the hardware cluster barrier (tuning key "cluster", off
+ * by default). Every
  * variant runs the same structure; results are identical to `gens` calls of
  * vf_gol_step. VF_ERR_CUDA if the grid cannot be co-resident. */
 vf_status vf_gol_run(vf_ctx* ctx, vf_variant v, uint32_t W, uint32_t H, int torus, uint8_t* state0_dev,
@@ -654,7 +658,11 @@ vf_status vf_checksum_i32(const int32_t* vals_dev, uint64_t n, long long* out_de
  * "persistent" = 1 runs the grouped kernels on a persistent grid (CTAs loop
  * over tiles), 0 gives every CTA one tile, -1 (default) = persistent except
  * for the app methods marked heavy (long bodies of varying length: collision
- * and N-body update, graph methods).
+ * and N-body update, graph methods); "cluster" = 1 lets vf_gol_run run
+ * grids of <= 2^17 cells in ONE thread-block cluster (state in distributed
+ * shared memory, hardware cluster barrier), 0 (default; measured faster on
+ * B200: a 16-SM cluster serialises 4 cells per thread) always uses the
+ * cooperative grid-barrier kernel.
  * VF_ERR_INVALID for unknown keys / values. */
 vf_status vf_set_tuning(const char* key, int value);
 /* Number of libvf kernel launches issued since load (for bench accounting). */

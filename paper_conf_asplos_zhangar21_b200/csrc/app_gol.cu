@@ -7,6 +7,7 @@
 // Object layout (16 B): { vTable* (8 B), u32 cell, u16 counter, u16 pad }.
 // counter = age (Alive) / dead_for (Dead): incremented by next(), reset to 0
 // when the cell switches to this object.
+#include <cooperative_groups.h>
 #include <cstring>
 
 #include "dispatch.cuh"
@@ -116,6 +117,14 @@ struct Step {
   const uint64_t* dead;
   __device__ __forceinline__ void pre(uint64_t c) const { nbr[c] = count_live(W, H, torus, prev, c); }
   __device__ __forceinline__ uint64_t ptr(uint64_t c) const { return grid[c]; }
+  // the body reads nbr[cell] (just written by pre) and the object's counter
+  __device__ __forceinline__ uint32_t warm(uint64_t c, uint64_t a) const {
+    uint32_t v, w;
+    asm volatile("ld.global.ca.u8 %0, [%1];" : "=r"(v) : "l"(nbr + c));
+    asm volatile("ld.global.ca.u32 %0, [%1];" : "=r"(w) : "l"(a + 8));
+    return v ^ w;
+  }
+  __device__ __forceinline__ uint64_t* ptr_base() const { return grid; }
   __device__ __forceinline__ void post(uint64_t c) const {
     const uint8_t s = next[c];
     if (s != prev[c]) {
@@ -247,6 +256,185 @@ __global__ void __launch_bounds__(kBlock) k_run_virtual(RunArgs r) {
   }
 }
 
+// Cluster variant (small grids, e.g. config 1's 256 x 256): ONE thread-block
+// cluster of C CTAs (up to 16, non-portable size) runs every generation. CTA r
+// keeps its block of rows of the state in shared memory (double-buffered);
+// neighbour rows owned by other CTAs are read through distributed shared
+// memory, and generations are separated by the hardware cluster barrier
+// (barrier.cluster, ~0.2 us, which also orders the DSMEM writes). The method
+// still writes its next state to global memory (its contract); the owning
+// thread reads its own write back into shared memory for the neighbours.
+constexpr int kClusterBlock = 1024;
+
+template <class R>
+__global__ void __launch_bounds__(kClusterBlock, 1) k_run_cluster(RunArgs r, DevTable tbl, uint32_t rows_per) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  namespace cg = cooperative_groups;
+  cg::cluster_group cluster = cg::this_cluster();
+  const uint32_t rank = cluster.block_rank();
+  const size_t tbytes = R::kNeedsTable ? (table_smem_dev(tbl.P) + 15) / 16 * 16 : 0;
+  if constexpr (R::kNeedsTable) R::stage(smem, tbl);
+  uint8_t* const sb0 = smem + tbytes;
+  uint8_t* const sb1 = smem + tbytes + (size_t)rows_per * r.W;
+  const uint32_t W = r.W, H = r.H;
+  const uint32_t y0 = rank * rows_per;
+  const uint32_t y1 = min(H, y0 + rows_per);
+  const uint32_t own = y1 > y0 ? (y1 - y0) * W : 0u;
+  // initial state of the owned rows
+  for (uint32_t k = threadIdx.x; k < own; k += kClusterBlock) sb0[k] = r.buf[0][(uint64_t)y0 * W + k];
+  cluster.sync();
+  uint32_t hint = 0;
+  for (uint32_t g = 0; g < r.gens; ++g) {
+    const uint8_t* cur = (g & 1) ? sb1 : sb0;
+    uint8_t* nxt_s = (g & 1) ? sb0 : sb1;
+    uint8_t* next = (g & 1) ? r.buf[0] : r.buf[1];
+    ArgBlob args{};
+    const vf_gol_next_args a{r.nbr, next};
+    *reinterpret_cast<vf_gol_next_args*>(args.b) = a;
+    const uint32_t iters = (own + kClusterBlock - 1) / kClusterBlock;  // CTA-uniform
+    for (uint32_t it = 0; it < iters; ++it) {
+      const uint32_t k = it * kClusterBlock + threadIdx.x;
+      const bool valid = k < own;
+      uint64_t c = 0, p = 0, ad = 0;
+      uint32_t t = kNF;
+      uint8_t prev_s = 0;
+      if (valid) {
+        const uint32_t y = y0 + k / W, x = k % W;
+        c = (uint64_t)y * W + x;
+        int n = 0;
+#pragma unroll
+        for (int dy = -1; dy <= 1; ++dy) {
+          int yy = (int)y + dy;
+          if (r.torus) yy = (yy + (int)H) % (int)H;
+          else if (yy < 0 || yy >= (int)H) continue;
+          const uint32_t owner = (uint32_t)yy / rows_per;
+          const uint8_t* row = (owner == rank ? const_cast<uint8_t*>(cur)
+                                              : cluster.map_shared_rank(const_cast<uint8_t*>(cur), owner)) +
+                               (size_t)((uint32_t)yy - owner * rows_per) * W;
+#pragma unroll
+          for (int dx = -1; dx <= 1; ++dx) {
+            if (dx == 0 && dy == 0) continue;
+            int xx = (int)x + dx;
+            if (r.torus) xx = (xx + (int)W) % (int)W;
+            else if (xx < 0 || xx >= (int)W) continue;
+            n += row[xx] == 1;
+          }
+        }
+        r.nbr[c] = (uint8_t)n;
+        prev_s = cur[k];
+        p = r.grid[c];
+      }
+      if (p) t = R::resolve(smem, tbl.P, p, ad, hint);
+      group_call<App, VF_GOL_NEXT>(t, ad, p, c, args, tbl);
+      if (valid) {
+        const uint8_t s = *(volatile const uint8_t*)(next + c);  // this thread's own write
+        if (s != prev_s) {
+          const uint64_t q = s ? r.alive[c] : r.dead[c];
+          r.grid[c] = q;
+          reinterpret_cast<Cell*>(strip(q))->counter = 0;
+        }
+        nxt_s[k] = s;
+      }
+    }
+    cluster.sync();
+  }
+}
+
+template <class R>
+__global__ void __launch_bounds__(kClusterBlock, 1) k_run_cluster_virtual(RunArgs r, DevTable tbl,
+                                                                        uint32_t rows_per) {
+  (void)tbl;
+  extern __shared__ __align__(16) unsigned char smem[];
+  namespace cg = cooperative_groups;
+  cg::cluster_group cluster = cg::this_cluster();
+  const uint32_t rank = cluster.block_rank();
+  uint8_t* const sb0 = smem;
+  uint8_t* const sb1 = smem + (size_t)rows_per * r.W;
+  const uint32_t W = r.W, H = r.H;
+  const uint32_t y0 = rank * rows_per;
+  const uint32_t y1 = min(H, y0 + rows_per);
+  const uint32_t own = y1 > y0 ? (y1 - y0) * W : 0u;
+  for (uint32_t k = threadIdx.x; k < own; k += kClusterBlock) sb0[k] = r.buf[0][(uint64_t)y0 * W + k];
+  cluster.sync();
+  for (uint32_t g = 0; g < r.gens; ++g) {
+    const uint8_t* cur = (g & 1) ? sb1 : sb0;
+    uint8_t* nxt_s = (g & 1) ? sb0 : sb1;
+    uint8_t* next = (g & 1) ? r.buf[0] : r.buf[1];
+    const vf_gol_next_args a{r.nbr, next};
+    for (uint32_t k = threadIdx.x; k < own; k += kClusterBlock) {
+      const uint32_t y = y0 + k / W, x = k % W;
+      const uint64_t c = (uint64_t)y * W + x;
+      int n = 0;
+#pragma unroll
+      for (int dy = -1; dy <= 1; ++dy) {
+        int yy = (int)y + dy;
+        if (r.torus) yy = (yy + (int)H) % (int)H;
+        else if (yy < 0 || yy >= (int)H) continue;
+        const uint32_t owner = (uint32_t)yy / rows_per;
+        const uint8_t* row = (owner == rank ? const_cast<uint8_t*>(cur)
+                                            : cluster.map_shared_rank(const_cast<uint8_t*>(cur), owner)) +
+                             (size_t)((uint32_t)yy - owner * rows_per) * W;
+#pragma unroll
+        for (int dx = -1; dx <= 1; ++dx) {
+          if (dx == 0 && dy == 0) continue;
+          int xx = (int)x + dx;
+          if (r.torus) xx = (xx + (int)W) % (int)W;
+          else if (xx < 0 || xx >= (int)W) continue;
+          n += row[xx] == 1;
+        }
+      }
+      r.nbr[c] = (uint8_t)n;
+      const uint8_t prev_s = cur[k];
+      const uint64_t p = r.grid[c];
+      if (p) reinterpret_cast<Cell*>(p)->next(a);  // the compiler's virtual call
+      const uint8_t s = *(volatile const uint8_t*)(next + c);
+      if (s != prev_s) {
+        const uint64_t q = s ? r.alive[c] : r.dead[c];
+        r.grid[c] = q;
+        reinterpret_cast<Cell*>(strip(q))->counter = 0;
+      }
+      nxt_s[k] = s;
+    }
+    cluster.sync();
+  }
+}
+
+// Launch one cluster of C CTAs if the grid's rows fit; returns
+// cudaErrorNotSupported (caller falls back to the grid-barrier kernels) if not.
+template <class K>
+static cudaError_t cluster_launch(K kern, const RunArgs& r, const DevTable& tbl, size_t table_bytes, cudaStream_t s) {
+  const uint64_t n = (uint64_t)r.W * r.H;
+  if (n > (1u << 17)) return cudaErrorNotSupported;  // bigger grids: the whole GPU, not one cluster
+  for (int C : {16, 8}) {
+    const uint32_t rows_per = (r.H + C - 1) / C;
+    const size_t sm = (table_bytes + 15) / 16 * 16 + 2 * (size_t)rows_per * r.W;
+    if (sm > 200 * 1024) continue;
+    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    if (C > 8) cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = dim3(C);
+    cfg.blockDim = dim3(kClusterBlock);
+    cfg.dynamicSmemBytes = sm;
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = C;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    int nclusters = 0;
+    if (cudaOccupancyMaxActiveClusters(&nclusters, (const void*)kern, &cfg) != cudaSuccess || nclusters < 1) {
+      cudaGetLastError();
+      continue;
+    }
+    const cudaError_t e = cudaLaunchKernelEx(&cfg, kern, r, tbl, rows_per);
+    note_launch();
+    return e;
+  }
+  return cudaErrorNotSupported;
+}
+
 template <class K>
 static cudaError_t coop_launch(K kern, uint64_t n, size_t sm, void** params, cudaStream_t s) {
   int occ = 0;
@@ -283,6 +471,23 @@ cudaError_t gol_run(int variant, uint32_t W, uint32_t H, int torus, uint8_t* buf
   gol::RunArgs r{W, H, torus, gens, {buf0, buf1}, nbr, grid, alive, dead, bar};
   DevTable t = tbl;
   void* params[2] = {&r, &t};
+  // small grids: one thread-block cluster, state in distributed shared memory
+  if (tuning().cluster != 0) {
+    cudaError_t ce = cudaErrorNotSupported;
+    switch (variant) {
+      case VF_CUDA:
+      case VF_SHAREDOA:
+        ce = gol::cluster_launch(gol::k_run_cluster_virtual<ResolveTP>, r, t, 0, s);
+        break;
+      case VF_COAL:
+        ce = gol::cluster_launch(gol::k_run_cluster<ResolveCOAL>, r, t, table_smem(tbl), s);
+        break;
+      case VF_TYPEPTR:
+        ce = gol::cluster_launch(gol::k_run_cluster<ResolveTP>, r, t, 0, s);
+        break;
+    }
+    if (ce != cudaErrorNotSupported) return ce;
+  }
   switch (variant) {
     case VF_CUDA:
     case VF_SHAREDOA:

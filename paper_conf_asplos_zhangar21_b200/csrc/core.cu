@@ -423,6 +423,9 @@ vf_status vf_set_tuning(const char* key, int value) {
   } else if (!strcmp(key, "persistent")) {
     if (value < -1 || value > 1) return VF_ERR_INVALID;
     tuning().persistent = value;
+  } else if (!strcmp(key, "cluster")) {
+    if (value < 0 || value > 1) return VF_ERR_INVALID;
+    tuning().cluster = value;
   } else {
     return VF_ERR_INVALID;
   }

@@ -22,6 +22,7 @@
 
 #include <new>
 #include <type_traits>
+#include <utility>
 
 #include "vf_internal.h"
 
@@ -1098,6 +1099,18 @@ cudaError_t verify_impl(int variant, const uint64_t* ptrs, uint64_t n, unsigned 
 //   __device__ void pre(uint64_t c) const; uint64_t ptr(uint64_t c) const;
 //   void post(uint64_t c) const;
 // ---------------------------------------------------------------------------
+// Optional Step hook `uint32_t warm(uint64_t c, uint64_t addr) const`: touch
+// (L1-allocating loads) what the method will read before the type groups run
+// one after another, so the second group's loads hit L1 (cf. warm_line).
+template <class S, class = void>
+struct HasWarm {
+  static constexpr bool value = false;
+};
+template <class S>
+struct HasWarm<S, std::void_t<decltype(std::declval<const S&>().warm(0ull, 0ull))>> {
+  static constexpr bool value = true;
+};
+
 template <class App, int M, class R, class Step>
 __global__ void __launch_bounds__(kBlock) k_step_grouped(uint64_t n, ArgBlob args, DevTable tbl, Step st) {
   extern __shared__ __align__(16) unsigned char smem[];
@@ -1114,7 +1127,14 @@ __global__ void __launch_bounds__(kBlock) k_step_grouped(uint64_t n, ArgBlob arg
       p = st.ptr(c);
     }
     if (p) t = R::resolve(smem, tbl.P, p, a, hint);
-    group_call<App, M>(t, a, p, c, args, tbl);
+    if constexpr (HasWarm<Step>::value) {
+      uint32_t sink = 0;
+      if (valid && t < (uint32_t)App::kTypes) sink = st.warm(c, a);
+      group_call<App, M>(t, a, p, c, args, tbl);
+      if (sink == 0x8BADF00Du && n == ~0ull) asm volatile("st.global.u32 [%0], %1;" ::"l"(st.ptr_base()), "r"(sink));
+    } else {
+      group_call<App, M>(t, a, p, c, args, tbl);
+    }
     if (valid) st.post(c);
   }
 }

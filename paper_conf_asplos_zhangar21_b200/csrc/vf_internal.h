@@ -93,6 +93,7 @@ struct Tuning {
   int regroup = 1;    // 1: CTA-level counting sort of each tile by type (k_dispatch_sorted)
   int call = 0;       // COAL / TypePointer: 0 grouped direct call, 1 indirect CALL via vFunc* table
   int persistent = -1; // grouped kernels: 1 persistent grid, 0 one tile per CTA, -1 app default (kHeavyMask)
+  int cluster = 0;     // vf_gol_run: 1 one thread-block cluster (state in DSMEM) when the grid fits
 };
 Tuning& tuning();
 

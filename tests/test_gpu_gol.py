@@ -72,9 +72,13 @@ def test_gol_cuda_graph_capture(ctx):
 @pytest.mark.parametrize("variant", VARIANTS)
 @pytest.mark.parametrize("W,H,gens,torus", [(256, 256, 100, False), (37, 23, 31, False), (64, 48, 25, True),
                                             (1024, 1024, 7, False)])
-def test_gol_persistent_run(ctx, variant, W, H, gens, torus):
-    """vf_gol_run: all generations in one cooperative launch (grid barrier between
-    generations; at 1024^2 each thread owns several cells) == the oracle."""
+@pytest.mark.parametrize("cluster", [1, 0])
+def test_gol_persistent_run(ctx, variant, W, H, gens, torus, cluster):
+    """vf_gol_run: all generations in one launch == the oracle. cluster = 1: grids
+    of <= 2^17 cells run in one thread-block cluster (DSMEM state rows); larger
+    grids and cluster = 0 use the cooperative grid-barrier kernel (at 1024^2 each
+    thread owns several cells)."""
+    vf.set_tuning("cluster", cluster)
     g0 = synth.soup(W, H, seed=43)
     st_ref, ctr_ref, _, _ = oracle.gol_run(W, H, g0, gens, torus)
     g = apps.Gol(ctx, W, H, g0, variant, torus)
@@ -88,3 +92,4 @@ def test_gol_persistent_run(ctx, variant, W, H, gens, torus):
     g2.run(gens // 2)
     g2.run(gens - gens // 2)
     assert np.array_equal(g2.current.cpu().numpy(), st_ref)
+    vf.set_tuning("cluster", 0)

@@ -97,9 +97,14 @@ def bench_gol(ctx, quick):
         record("gol", "256x256, 100 gens (CUDA graph of 100 generations)", v, W * H, ms, 14, "GB/s", "l2/latency",
                dict(ms_per_gen_eager=ms_eager, ms_per_gen_eager_unfused=ms_unfused), cpu)
         del graph
+        vf.set_tuning("cluster", 1)
         ms_run = ev_time(lambda: g.run(gens), 5) / gens
-        record("gol-run", "256x256, 100 gens in one persistent cooperative launch (vf_gol_run)", v, W * H, ms_run,
-               14, "GB/s", "l2/latency", None, cpu)
+        vf.set_tuning("cluster", 0)
+        record("gol-cluster", "256x256, 100 gens in ONE thread-block cluster launch (vf_gol_run, DSMEM state)", v,
+               W * H, ms_run, 14, "GB/s", "l2/latency", None, cpu)
+        ms_run = ev_time(lambda: g.run(gens), 5) / gens
+        record("gol-coop", "256x256, 100 gens in one cooperative grid-barrier launch (vf_gol_run, cluster=0)", v,
+               W * H, ms_run, 14, "GB/s", "l2/latency", None, cpu)
         del g
     ctx.reset()
 
