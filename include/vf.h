@@ -531,6 +531,17 @@ vf_status vf_dispatch_concord(vf_ctx* ctx, uint32_t app, uint32_t method, const 
 vf_status vf_dispatch(vf_ctx* ctx, vf_variant v, uint32_t app, uint32_t method,
                       const uint64_t* objs_dev, uint64_t n, const void* args, size_t args_bytes,
                       void* stream);
+/* Dispatch from a HOST pointer array (the end-to-end path): objs_host (n
+ * pointers; pinned memory for full PCIe bandwidth) is copied in chunks of
+ * `chunk` pointers (0 = 2^22) into staging_dev (caller-owned device buffer of
+ * n u64) on a ctx-internal copy stream, and every chunk is dispatched on
+ * `stream` as soon as its copy has landed, so the transfer overlaps the
+ * calls. Same semantics as vf_dispatch over the copied array. Asynchronous:
+ * objs_host must stay valid and unchanged until `stream` has passed this
+ * call; staging_dev is overwritten only after earlier work on `stream`. */
+vf_status vf_dispatch_host(vf_ctx* ctx, vf_variant v, uint32_t app, uint32_t method, const uint64_t* objs_host,
+                           uint64_t n, const void* args, size_t args_bytes, uint64_t* staging_dev, uint64_t chunk,
+                           void* stream);
 
 /* ---- app helpers (non-virtual phases) ---------------------------------- */
 /* GOL / GEN step (1): nbr_dev[c] = neighbours of cell c whose state is 1

@@ -130,6 +130,9 @@ struct vf_ctx {
   std::vector<HeapBatch> heap;
   std::vector<uint64_t> type_count[VF_APP_COUNT];  // live objects per (app, type)
   size_t gran = 2u << 20;
+  // vf_dispatch_host: copy stream + one event per chunk (created on first use)
+  cudaStream_t copy_stream = nullptr;
+  std::vector<cudaEvent_t> chunk_events;
 };
 
 namespace {
@@ -539,6 +542,8 @@ void vf_destroy(vf_ctx* c) {
     cudaFree(t.d_type);
     cudaFree(t.d_vptr);
   }
+  for (cudaEvent_t e : c->chunk_events) cudaEventDestroy(e);
+  if (c->copy_stream) cudaStreamDestroy(c->copy_stream);
   delete c;
 }
 
@@ -723,6 +728,39 @@ vf_status vf_dispatch(vf_ctx* c, vf_variant v, uint32_t app, uint32_t method,
   if (e == cudaErrorNotSupported)
     return fail(c, VF_ERR_UNSUPPORTED, "app %s has no embedded type tag (Concord)", ops->name);
   CUDA_TRY(c, e);
+  return VF_OK;
+}
+
+vf_status vf_dispatch_host(vf_ctx* c, vf_variant v, uint32_t app, uint32_t method, const uint64_t* objs_host,
+                           uint64_t n, const void* args, size_t args_bytes, uint64_t* staging_dev, uint64_t chunk,
+                           void* stream) {
+  vf_status st = check_app(c, app);
+  if (st) return st;
+  if (!n) return VF_OK;
+  if (!objs_host || !staging_dev) return fail(c, VF_ERR_INVALID, "null host array or staging buffer");
+  if ((st = set_device(c))) return st;
+  if (!chunk) chunk = 1ull << 22;
+  const uint64_t nchunks = (n + chunk - 1) / chunk;
+  if (!c->copy_stream) CUDA_TRY(c, cudaStreamCreateWithFlags(&c->copy_stream, cudaStreamNonBlocking));
+  while (c->chunk_events.size() < nchunks + 1) {
+    cudaEvent_t e;
+    CUDA_TRY(c, cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    c->chunk_events.push_back(e);
+  }
+  cudaStream_t us = S(stream);
+  // the staging buffer may still be read by earlier work on `stream`
+  CUDA_TRY(c, cudaEventRecord(c->chunk_events[nchunks], us));
+  CUDA_TRY(c, cudaStreamWaitEvent(c->copy_stream, c->chunk_events[nchunks], 0));
+  for (uint64_t k = 0; k < nchunks; ++k) {
+    const uint64_t off = k * chunk, m = n - off < chunk ? n - off : chunk;
+    CUDA_TRY(c, cudaMemcpyAsync(staging_dev + off, objs_host + off, 8 * m, cudaMemcpyHostToDevice, c->copy_stream));
+    CUDA_TRY(c, cudaEventRecord(c->chunk_events[k], c->copy_stream));
+  }
+  for (uint64_t k = 0; k < nchunks; ++k) {
+    const uint64_t off = k * chunk, m = n - off < chunk ? n - off : chunk;
+    CUDA_TRY(c, cudaStreamWaitEvent(us, c->chunk_events[k], 0));
+    if ((st = vf_dispatch(c, v, app, method, staging_dev + off, m, args, args_bytes, stream))) return st;
+  }
   return VF_OK;
 }
 

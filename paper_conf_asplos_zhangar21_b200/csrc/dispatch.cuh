@@ -951,14 +951,19 @@ cudaError_t launch_grouped_tuned(const uint64_t* objs, uint64_t n, const ArgBlob
       return launch_sorted<App, M, R, App::kUnrollSorted, App::kPrefetch>(objs, n, args, tbl, s);
     return launch_grouped<App, M, R, App::kUnroll, App::kPrefetch>(objs, n, args, tbl, s);
   } else {
-  // Measured on B200 (config 2, 2^26 objects): with the per-tile type sort,
-  // 2 objects per thread + L1 warm-up is best up to ~16 live types; with >= 24
-  // live types (the sort leaves ~half-warp groups) 4 objects per thread
-  // without warm-up wins. Without the sort, >= 24 types prefer 1 object/thread.
+  // Measured on B200 (config 2, 2^26 objects, profiles/sweep_knobs_r1.md):
+  // with the per-tile type sort and the next tile's pointers in flight, the
+  // L1 warm-up (prefetch 2; config 2's app default) wins at every type
+  // count, also at >= 24 live types where it used to lose; 2 objects per thread up
+  // to ~16 live types; with >= 24 live types (the sort leaves ~half-warp
+  // groups) TypePointer prefers 4 objects per thread, COAL (whose smem search
+  // adds registers) stays at 2. Without the sort, >= 24 types prefer 1.
   const bool rg = tu.regroup != 0 && App::kTypes > 1;
   const bool many = tbl.active_types >= 24;
-  const int u = tu.unroll > 0 ? tu.unroll : rg ? (many ? 4 : App::kUnrollSorted) : (many ? 1 : App::kUnroll);
-  const int pf = tu.prefetch >= 0 ? tu.prefetch : (rg && many) ? 0 : App::kPrefetch;
+  const int u = tu.unroll > 0 ? tu.unroll
+                : rg ? (many ? (R::kNeedsTable ? 2 : 4) : App::kUnrollSorted)
+                     : (many ? 1 : App::kUnroll);
+  const int pf = tu.prefetch >= 0 ? tu.prefetch : (rg && many) ? 2 : App::kPrefetch;
   if (u >= 4) return launch_grouped_pf<App, M, R, 4>(pf, objs, n, args, tbl, s);
   if (u == 2) return launch_grouped_pf<App, M, R, 2>(pf, objs, n, args, tbl, s);
   return launch_grouped_pf<App, M, R, 1>(pf, objs, n, args, tbl, s);

@@ -39,7 +39,7 @@ SYMBOLS = [
     "vf_regions", "vf_type_vptrs", "vf_resolve", "vf_verify_types", "vf_dispatch_cuda",
     "vf_dispatch_sharedoa", "vf_dispatch_coal", "vf_dispatch_typeptr", "vf_dispatch",
     "vf_gol_neighbors", "vf_gol_swap", "vf_gen_swap", "vf_checksum_i32", "vf_launch_count", "vf_set_tuning",
-    "vf_graph_bfs_init", "vf_iota_u32", "vf_fill_f32", "vf_ray_render", "vf_gol_step", "vf_gen_step", "vf_gol_run",
+    "vf_graph_bfs_init", "vf_iota_u32", "vf_fill_f32", "vf_ray_render", "vf_gol_step", "vf_gen_step", "vf_gol_run", "vf_dispatch_host",
     "vf_dispatch_concord", "vf_micro_branch", "vf_collide_tmp_words", "vf_collide_grid",
 ]
 APP_RAY = 4
@@ -271,6 +271,7 @@ def lib(required: bool = True):
         "vf_ray_render": (I, [P, I, P, U32, U32, U32, U32, U32, P, P, P, P, P]),
         "vf_gol_step": (I, [P, I, U32, U32, I, P, P, P, P, P, P, P]),
         "vf_gol_run": (I, [P, I, U32, U32, I, P, P, P, P, P, P, U32, P, P]),
+        "vf_dispatch_host": (I, [P, I, U32, U32, P, U64, P, ctypes.c_size_t, P, U64, P]),
         "vf_dispatch_concord": (I, [P, U32, U32, P, U64, P, ctypes.c_size_t, P]),
         "vf_micro_branch": (I, [U64, U32, I, U64, U32, P, P]),
         "vf_collide_tmp_words": (U64, [U32, U32]),
@@ -441,6 +442,13 @@ class Ctx:
         n = objs.numel() if n is None else n
         self._check(self.L.vf_dispatch(self.h, variant, app, method, _ptr(objs), n, a, ab,
                                        _stream(stream)), "dispatch")
+
+    def dispatch_host(self, variant, app, method, objs_host, staging, args=None, chunk=0, stream=None):
+        """vf_dispatch_host: objs_host = pinned CPU int64 tensor of object pointers,
+        staging = device int64 tensor of the same length (overwritten)."""
+        a, ab = _args(args)
+        self._check(self.L.vf_dispatch_host(self.h, variant, app, method, objs_host.data_ptr(), objs_host.numel(),
+                                            a, ab, _ptr(staging), chunk, _stream(stream)), "dispatch_host")
 
     def dispatch_raw(self, variant, app, method, objs_ptr: int, n: int, args=None, stream=None):
         """Same as dispatch() with a raw device pointer (hot loops avoid tensor overhead)."""

@@ -253,3 +253,24 @@ def test_concord_unsupported_without_tag(ctx):
     with pytest.raises(vf.VFError) as e:
         ctx.dispatch(vf.CONCORD, vf.APP_GOL, vf.GOL_NEXT, g.grid, g.args[0])
     assert e.value.status == 7
+
+
+@pytest.mark.parametrize("variant", ["cuda", "sharedoa", "coal", "typeptr"])
+@pytest.mark.parametrize("chunk", [0, 1000, 4096 * 3 + 5])
+def test_dispatch_host_matches_closed_form(variant, chunk):
+    """vf_dispatch_host (chunked H2D overlapped with the calls) == the closed form
+    val_i = init_i + R (t_i + 1), for chunk sizes that leave ragged tails."""
+    import torch
+    c = vf.Ctx(0, cuda_heap_bytes=1 << 30)
+    n, T, R = 4096 * 5 + 77, 4, 3
+    types = synth.micro_types(n, T, "random", seed=9)
+    init = synth.micro_init(n, seed=9)
+    m = apps.Micro(c, n, T, variant=variant, types_np=types, init_np=init)
+    host = m.objs.cpu().pin_memory()
+    staging = torch.empty_like(m.objs)
+    for _ in range(R):
+        c.dispatch_host(m.v, vf.APP_MICRO, vf.MICRO_APPLY, host, staging, chunk=chunk)
+    got = m.values().cpu().numpy()
+    assert np.array_equal(got, init + R * (types.astype(np.int32) + 1))
+    assert torch.equal(staging, m.objs)
+    c.close()
