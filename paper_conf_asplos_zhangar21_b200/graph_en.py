@@ -31,6 +31,13 @@ from .graph import work_entries
 HUB = 3  # vertex type id of Hub (deg >= 256)
 
 
+def reverse_arcs(col: torch.Tensor) -> torch.Tensor:
+    """rev[k] = index of the reverse arc (col[k] -> v) of arc k = (v -> col[k]) in
+    a symmetric CSR with sorted rows: a stable sort of the arcs by target lists,
+    for each v, the arcs (u -> v) in ascending u, i.e. in the order of v's row."""
+    return torch.argsort(col, stable=True)
+
+
 class GraphEN:
     def __init__(self, ctx: vf.Ctx, offs: np.ndarray, col: np.ndarray, variant: str = "typeptr", chunk: int = 256):
         self.ctx, self.variant = ctx, variant
@@ -68,7 +75,7 @@ class GraphEN:
         self.etypes = etypes
         del ector
         # in-edges of v in ascending source order: the arcs (u -> v) sorted stably by v
-        rev = torch.argsort(col_t, stable=True)
+        rev = reverse_arcs(col_t)
         self.in_edges = self.out_edges[rev].contiguous()
         del rev, col_t
         # ---- nested edge-call resolver (COAL table / TypePointer tag / vTable* fallback)
