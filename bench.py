@@ -153,6 +153,17 @@ def oracle_micro_sample(args, n_s, reps, threads):
 
 
 # --------------------------------------------------------------------------- reference arm
+def workload_config(args, world):
+    """The workload both arms measure (the reference arm times a bounded sample
+    of it on the host; its cpu_baseline.sample says which)."""
+    return {"workload": f"micro: n={args.n} objects/GPU x T={args.T} types, {args.order} order, "
+                        f"1 virtual apply() per object per step",
+            "variant": args.variant, "n": args.n, "T": args.T, "order": args.order,
+            "seed": args.seed, "object_bytes": 16,
+            "l2": "inputs larger than L2 (1.5 GiB objects+pointers per GPU >> 126 MB)",
+            "parallelism": f"dp{world} (independent object shards)"}
+
+
 def run_reference(args, rank, world):
     if rank != 0:
         return
@@ -170,8 +181,7 @@ def run_reference(args, rank, world):
            "value": v, "unit": "calls/s", "n_gpus": args.gpus, "steps": k, "warmup": args.warmup,
            "ms_per_step": 1e3 * tot / k, "higher_is_better": True, "scaling": "weak",
            "vs_baseline": None, "dtype": "int32", "data": "synthetic",
-           "config": {"workload": f"micro n={args.n} T={args.T} order={args.order} (CPU sample n={n_s})",
-                      "n": args.n, "T": args.T, "order": args.order},
+           "config": workload_config(args, world),
            "cpu_baseline": {"value": v, "unit": "calls/s", "cores": threads, "kind": "oracle",
                             "sample": f"{n_s} objects per step ({args.order}, T={args.T}), one pass, "
                                       f"OpenMP {threads} threads, {cpu_model()}"},
@@ -366,12 +376,7 @@ def run_ours(args, rank, world, local):
                "unit": "calls/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
                "ms_per_step": step_ms, "higher_is_better": True, "scaling": "weak",
                "vs_baseline": None, "dtype": "int32", "data": "synthetic",
-               "config": {"workload": f"micro: n={n} objects/GPU x T={args.T} types, {args.order} order, "
-                                      f"1 virtual apply() per object per step",
-                          "variant": args.variant, "n": n, "T": args.T, "order": args.order,
-                          "seed": args.seed, "object_bytes": 16,
-                          "l2": "inputs larger than L2 (1.5 GiB objects+pointers per GPU >> 126 MB)",
-                          "parallelism": f"dp{world} (independent object shards)"},
+               "config": workload_config(args, world),
                "gpu_launches": launches, "parity_sample_ok": ok, "roofline": roof, "clocks": clk,
                "e2e": e2e, "cpu_baseline": cpu, "variants": results}
         print(json.dumps(out), flush=True)
