@@ -139,6 +139,7 @@ struct App {
   static constexpr int kUnrollSorted = 2;
   static constexpr int kPrefetch = 2;
   static constexpr uint32_t kHeavyMask = 0x1Fu;  // one tile per CTA (dispatch.cuh grid_cap)
+  static constexpr int kMinBlocks = 4;           // <= 64 registers: random gathers need resident warps
   using Base = Vertex;
   template <int K>
   using Type = VertexK<K>;
