@@ -105,3 +105,25 @@ def test_graph_en_f6_fixture(ctx):
         label, _, _, _ = g.cc()
         assert list(label.cpu().numpy()) == [0, 0, 0, 0, 4, 4]
         torch.cuda.synchronize()
+
+
+@pytest.mark.parametrize("variant", VARIANTS)
+def test_graph_en_degenerate_graphs(ctx, variant):
+    """No edges at all (every vertex dangling: PageRank stays uniform), and a
+    single edge plus isolated vertices: same results as the oracle."""
+    for V, edges in ((5, []), (6, [(2, 4)])):
+        offs, col = synth.csr_from_edges(V, edges)
+        types = synth.vertex_types(offs)
+        g = GraphEN(ctx, offs, col, variant)
+        assert g.A == 2 * len(edges)
+        d_ref, lv_ref, _, _, _ = oracle.graph_en_bfs(offs, col, types, 2)
+        depth, levels, _ = g.bfs(2)
+        assert np.array_equal(depth.cpu().numpy(), d_ref) and levels == lv_ref
+        l_ref, it_ref, _, _, _ = oracle.graph_en_cc(offs, col, types)
+        label, iters, _, _ = g.cc()
+        assert np.array_equal(label.cpu().numpy().view(np.uint32), l_ref) and iters == it_ref
+        r_ref, _ = oracle.graph_en_pr(offs, col, types, iters=7)
+        rank, _, _ = g.pagerank(7)
+        np.testing.assert_allclose(rank.cpu().numpy(), r_ref, rtol=1e-6, atol=0)
+        if not edges:
+            np.testing.assert_allclose(r_ref, 1.0 / V, rtol=1e-6)
