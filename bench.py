@@ -360,7 +360,9 @@ def run_ours(args, rank, world, local):
     peak_src = "MEASURED_PEAKS.json hbm_gbs (copy, burst), of measured"
     if not hbm:  # file absent on this box: the profiling guide's stated fallback
         hbm, peak_src = 6650.0, "B200_PROFILING.md fallback 6.65 TB/s (MEASURED_PEAKS.json absent), of fallback"
-    kern = f"k_dispatch_grouped<micro,apply,{'ResolveTP' if args.variant == 'typeptr' else 'ResolveCOAL'}>" \
+    # the library's default for these variants: the type-sorted tile kernel
+    # (vf_set_tuning "regroup" = 1), as in the ncu launch list (profiles/)
+    kern = f"k_dispatch_sorted<micro,apply,{'ResolveTP' if args.variant == 'typeptr' else 'ResolveCOAL'}>" \
         if args.variant in ("coal", "typeptr") else "k_dispatch_virtual<micro,apply>"
     achieved = ALG_BYTES_PER_CALL * n / (step_ms / 1e3) / 1e9
     tr = ncu_traffic(f"micro_{args.variant}_T{args.T}_{args.order}")
