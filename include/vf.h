@@ -269,10 +269,16 @@ enum {
                               iterate); *changed = 1 if it is below label_in[v]          */
   VF_GRAPH_PR_CONTRIB = 3, /* chunk 0 only: contrib[v] = deg ? rank_in[v]/deg : 0 (fp64);
                               deg-0 vertices add rank_in[v] to *dangling                 */
-  VF_GRAPH_PR_UPDATE = 4   /* rank_out[v] = (float)(base + d*(sum_{N(v)} contrib +
+  VF_GRAPH_PR_UPDATE = 4,  /* rank_out[v] = (float)(base + d*(sum_{N(v)} contrib +
                               *dangling / Vd)); a multi-chunk vertex writes its chunk sum
                               to partial[i]; the last chunk to finish (counter[v]) sums
                               the partials in chunk order and resets counter[v] to 0    */
+  VF_GRAPH_BFS_PROBE_BITS = 5 /* bottom-up over a frontier BITMAP (multi-GPU, SURVEY §8e:
+                              the per-level exchange is an all-gather of bitmap slices):
+                              an unvisited vertex v with a neighbour u whose bit is set in
+                              frontier_bits takes depth level+1 (atomicCAS), sets bit v of
+                              next_bits (atomicOr) and *next_count = 1. Args:
+                              vf_graph_bfs_bits_args                                     */
 };
 typedef struct {
   const uint64_t* offs_dev;
@@ -286,6 +292,19 @@ typedef struct {
   int32_t level;
   uint32_t C;                  /* edges per chunk (>= 1)                           */
 } vf_graph_bfs_args;
+/* VF_GRAPH_BFS_PROBE_BITS: bit v of a bitmap is word v >> 5, bit v & 31 (u32 words). */
+typedef struct {
+  const uint64_t* offs_dev;
+  const uint32_t* col_dev;
+  int32_t* depth_dev;          /* read + written for the dispatched (owned) vertices only */
+  const uint32_t* frontier_dev;/* ceil(V/32) words: vertices at depth `level`            */
+  uint32_t* next_dev;          /* ceil(V/32) words: owned vertices that joined level+1;
+                                  the caller zeroes the owned words before the call     */
+  const uint32_t* chunk_dev;
+  uint32_t* next_count_dev;
+  int32_t level;
+  uint32_t C;
+} vf_graph_bfs_bits_args;
 typedef struct {
   const uint64_t* offs_dev;
   const uint32_t* col_dev;
@@ -469,11 +488,28 @@ vf_status vf_alloc_typed(vf_ctx* ctx, uint32_t app, uint32_t type_id, uint64_t c
                          const void* ctor_args_dev, uint32_t ctor_arg_bytes,
                          uint64_t* out_ptrs_dev, int tag, void* stream);
 /* Batched: object i is of class (app, type_ids_dev[i]) and takes the next
- * slot of its type's arena in index order (allocation order = index order). */
+ * slot of its type's arena in index order (allocation order = index order).
+ * The slot of object i is its rank among the objects of its type with a
+ * smaller index: a device prefix count (per-chunk type histograms, a per-type
+ * scan, then a placement pass); only the per-type totals (ntypes x 8 B) come
+ * back to the host, which maps the regions. The app must have <= 32 types
+ * (VF_ERR_TOO_MANY_TYPES); a type id >= ntypes -> VF_ERR_INVALID. Synchronises
+ * `stream`; the range table is republished as a NEW device version (kernels
+ * still running on other streams keep reading the old one, which is freed at
+ * vf_reset / vf_destroy). */
 vf_status vf_alloc_typed_batch(vf_ctx* ctx, uint32_t app, const uint32_t* type_ids_dev,
                                uint64_t count, const void* ctor_args_dev,
                                uint32_t ctor_arg_bytes, uint64_t* out_ptrs_dev, int tag,
                                void* stream);
+/* cuda_packed (SURVEY §7 "A fair CUDA baseline", a sensitivity point for the
+ * CUDA baseline): object i of class (app, type_ids_dev[i]) is placement-new'd
+ * at slab + i * stride of ONE cudaMalloc'd index-ordered slab (stride = the
+ * app's largest object rounded to 16 B): embedded vTable*, no type grouping,
+ * no heap scatter. Dispatch it with VF_CUDA. Not in the range table. Freed at
+ * vf_reset / vf_destroy. */
+vf_status vf_alloc_packed(vf_ctx* ctx, uint32_t app, const uint32_t* type_ids_dev, uint64_t count,
+                          const void* ctor_args_dev, uint32_t ctor_arg_bytes, uint64_t* out_ptrs_dev,
+                          void* stream);
 /* CUDA baseline: device-heap `new` of class (app, type_ids_dev[i]) per object
  * in a kernel. tag = 1 additionally tags the
  * returned pointers (TypePointer on the default CUDA allocator, §8.2
@@ -588,6 +624,17 @@ vf_status vf_gen_step(vf_ctx* ctx, vf_variant v, uint32_t W, uint32_t H, int tor
                       uint8_t* state_next_dev, uint8_t* nbr_dev, uint64_t* grid_dev, const uint64_t* dead_dev,
                       const uint64_t* alive_dev, const uint64_t* dying_dev, uint32_t born_mask,
                       uint32_t survive_mask, uint32_t C, void* stream);
+/* The same generation restricted to the row slab [row0, row0 + nrows) (multi-GPU
+ * row slabs): neighbours of the slab's cells are read from
+ * state_prev rows row0-1 and row0+nrows (the halo rows, torus-wrapped when
+ * torus != 0), which the caller keeps current; only the slab's cells (and their
+ * grid_dev / nbr_dev / state_next_dev entries and objects) are touched. W*H <
+ * 2^32. VF_ERR_INVALID if the slab leaves [0, H). vf_gen_step = rows [0, H). */
+vf_status vf_gen_step_rows(vf_ctx* ctx, vf_variant v, uint32_t W, uint32_t H, int torus, uint32_t row0,
+                           uint32_t nrows, const uint8_t* state_prev_dev, uint8_t* state_next_dev,
+                           uint8_t* nbr_dev, uint64_t* grid_dev, const uint64_t* dead_dev, const uint64_t* alive_dev,
+                           const uint64_t* dying_dev, uint32_t born_mask, uint32_t survive_mask, uint32_t C,
+                           void* stream);
 
 /* Config 3 ray tracer (readings G24, G25): render rows [row0, row0+nrows) of
  * a W x H image over S shapes of VF_APP_RAY (type ids 0 Plane, 1 Sphere,

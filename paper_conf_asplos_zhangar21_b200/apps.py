@@ -98,9 +98,9 @@ class Gol:
         N = W * H
         self.N = N
         cells = torch.arange(N, dtype=torch.int32, device=dev)
-        if variant == "cuda":
-            self.alive = ctx.alloc_cuda(vf.APP_GOL, torch.ones(N, dtype=torch.int32, device=dev), cells)
-            self.dead = ctx.alloc_cuda(vf.APP_GOL, torch.zeros(N, dtype=torch.int32, device=dev), cells)
+        if variant in ("cuda", "cuda_packed"):
+            self.alive = ctx.alloc_for(variant, vf.APP_GOL, torch.ones(N, dtype=torch.int32, device=dev), cells)
+            self.dead = ctx.alloc_for(variant, vf.APP_GOL, torch.zeros(N, dtype=torch.int32, device=dev), cells)
         else:
             tag = variant == "typeptr"
             self.alive = ctx.alloc_typed(vf.APP_GOL, 1, N, cells, tag=tag)
@@ -159,30 +159,46 @@ def rule_masks(born: str, survive: str):
 
 class Gen:
     """Config 5 GEN: Generations CA B/S/C over polymorphic Dead / Alive / Dying cells
-    (Table 2, reading G15). Same three steps per generation as Gol."""
+    (Table 2, reading G15). Same three steps per generation as Gol.
+
+    Multi-GPU: row slabs. Rank r owns rows [r0, r1) (objects for
+    its cells only) and runs vf_gen_step_rows on them; after every generation
+    the boundary rows go to the neighbour slabs (exchange.HaloRows,
+    batch_isend_irecv of one W-byte row each way)."""
 
     def __init__(self, ctx: vf.Ctx, W: int, H: int, state0, variant: str = "typeptr",
-                 born: str = "2", survive: str = "345", C: int = 4, torus: bool = False):
+                 born: str = "2", survive: str = "345", C: int = 4, torus: bool = False,
+                 rank: int = 0, world: int = 1, group=None):
+        from . import exchange
         self.ctx, self.W, self.H, self.variant, self.torus = ctx, W, H, variant, torus
         self.v = vf.VARIANTS[variant]
         dev = _dev(ctx.device)
         N = W * H
         self.N = N
-        cells = torch.arange(N, dtype=torch.int32, device=dev)
+        self.rank, self.world = rank, world
+        self.halo = exchange.HaloRows(W, H, rank, world, torus, group)
+        self.r0, self.r1 = self.halo.r0, self.halo.r1
+        lo, hi = self.r0 * W, self.r1 * W
+        self.lo, self.hi = lo, hi
+        cells = torch.arange(lo, hi, dtype=torch.int32, device=dev)
         objs = []
         for t in range(3):
-            if variant == "cuda":
-                objs.append(ctx.alloc_cuda(vf.APP_GEN, torch.full((N,), t, dtype=torch.int32, device=dev), cells))
+            o = torch.zeros(N, dtype=torch.int64, device=dev)
+            if variant in ("cuda", "cuda_packed"):
+                o[lo:hi] = ctx.alloc_for(variant, vf.APP_GEN, torch.full((hi - lo,), t, dtype=torch.int32, device=dev),
+                                         cells)
             else:
-                objs.append(ctx.alloc_typed(vf.APP_GEN, t, N, cells, tag=(variant == "typeptr")))
+                o[lo:hi] = ctx.alloc_typed(vf.APP_GEN, t, hi - lo, cells, tag=(variant == "typeptr"))
+            objs.append(o)
         self.dead, self.alive, self.dying = objs
         self.grid = self.dead.clone()
-        s0 = torch.from_numpy(np.ascontiguousarray(state0, dtype=np.uint8)).to(dev)
-        zeros = torch.zeros(N, dtype=torch.uint8, device=dev)
-        vf.gen_swap(ctx, zeros, s0, self.grid, self.dead, self.alive, self.dying)
+        s0 = torch.from_numpy(np.ascontiguousarray(state0, dtype=np.uint8).reshape(-1)).to(dev)
+        zeros = torch.zeros(hi - lo, dtype=torch.uint8, device=dev)
+        vf.gen_swap(ctx, zeros, s0[lo:hi], self.grid[lo:hi], self.dead[lo:hi], self.alive[lo:hi],
+                    self.dying[lo:hi])
         self.state = s0.clone()
-        self.next = torch.empty_like(self.state)
-        self.nbr = torch.empty_like(self.state)
+        self.next = self.state.clone()
+        self.nbr = torch.zeros_like(self.state)
         bm, sm = rule_masks(born, survive)
         self.rule = (bm, sm, C)
         self.args = [vf.gen_next_args(self.nbr.data_ptr(), self.next.data_ptr(), bm, sm, C),
@@ -190,15 +206,21 @@ class Gen:
         self.parity = 0
         torch.cuda.synchronize(dev)
 
+    @property
+    def calls_per_gen(self):
+        return self.hi - self.lo
+
     def gen(self, stream=None, fused: bool = True):
         cur, nxt = (self.state, self.next) if self.parity == 0 else (self.next, self.state)
         if fused:
-            vf.gen_step(self.ctx, self.v, self.W, self.H, self.torus, cur, nxt, self.nbr, self.grid, self.dead,
-                        self.alive, self.dying, *self.rule, stream)
+            vf.gen_step_rows(self.ctx, self.v, self.W, self.H, self.torus, self.r0, self.r1 - self.r0, cur, nxt,
+                             self.nbr, self.grid, self.dead, self.alive, self.dying, *self.rule, stream)
         else:
+            assert self.world == 1, "the unfused form is single-GPU"
             vf.gol_neighbors(self.W, self.H, cur, self.nbr, self.torus, stream)
             self.ctx.dispatch(self.v, vf.APP_GEN, vf.GEN_NEXT, self.grid, self.args[self.parity], stream=stream)
             vf.gen_swap(self.ctx, cur, nxt, self.grid, self.dead, self.alive, self.dying, stream)
+        self.halo.exchange(nxt)
         self.parity ^= 1
 
     @property
@@ -206,7 +228,9 @@ class Gen:
         return self.state if self.parity == 0 else self.next
 
     def counters(self):
-        ctr = torch.empty(self.N, dtype=torch.int16, device=self.grid.device)
-        typ = torch.empty(self.N, dtype=torch.uint8, device=self.grid.device)
-        self.ctx.dispatch(self.v, vf.APP_GEN, vf.GEN_GET, self.grid, vf.gen_get_args(ctr.data_ptr(), typ.data_ptr()))
+        """(counter, type) per cell; only the owned rows [r0, r1) are written (others 0)."""
+        ctr = torch.zeros(self.N, dtype=torch.int16, device=self.grid.device)
+        typ = torch.zeros(self.N, dtype=torch.uint8, device=self.grid.device)
+        self.ctx.dispatch(self.v, vf.APP_GEN, vf.GEN_GET, self.grid[self.lo:self.hi],
+                          vf.gen_get_args(ctr.data_ptr(), typ.data_ptr()))
         return ctr, typ

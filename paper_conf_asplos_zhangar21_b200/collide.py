@@ -19,8 +19,8 @@ import ctypes
 import numpy as np
 import torch
 
-from . import vf
-from .graph import allgather_block, block_range
+from . import exchange as xc, vf
+from .exchange import block_range
 
 
 class Collide:
@@ -40,16 +40,16 @@ class Collide:
         ctor[:, 1:] = np.ascontiguousarray(sys_["vel"][own, :3], dtype=np.float32).view(np.uint32)
         tt = torch.from_numpy(sys_["types"][own].astype(np.int32)).to(dev)
         ct = torch.from_numpy(ctor.view(np.int32)).to(dev)
-        if variant == "cuda":
-            self.objs = ctx.alloc_cuda(vf.APP_COLLIDE, tt, ct)
-        else:
-            self.objs = ctx.alloc_typed_batch(vf.APP_COLLIDE, tt, ct, tag=(variant == "typeptr"))
+        self.objs = ctx.alloc_for(variant, vf.APP_COLLIDE, tt, ct)
         f4 = dict(dtype=torch.float32, device=dev)
-        self.P = torch.from_numpy(np.ascontiguousarray(sys_["pos"], dtype=np.float32)).to(dev)
-        self.Pm = torch.zeros((N, 4), **f4)
-        self.Vm = torch.zeros((N, 4), **f4)
+        blk = dict(n=N, per=self.per, rank=rank, world=world, device=dev, group=group)
+        self._P = xc.BlockArray(dtype=torch.float32, rest=(4,), fill=0.0, **blk)
+        self._P.view.copy_(torch.from_numpy(np.ascontiguousarray(sys_["pos"], dtype=np.float32)))
+        self._Pm = xc.BlockArray(dtype=torch.float32, rest=(4,), fill=0.0, **blk)
+        self._Vm = xc.BlockArray(dtype=torch.float32, rest=(4,), fill=0.0, **blk)
+        self._near = xc.BlockArray(dtype=torch.int32, fill=-1, **blk)
+        self.P, self.Pm, self.Vm, self.near = self._P.view, self._Pm.view, self._Vm.view, self._near.view
         self.Ps = torch.zeros((max(N, 1), 4), **f4)
-        self.near = torch.full((N,), -1, dtype=torch.int32, device=dev)
         ncell = self.G ** 3
         u32 = dict(dtype=torch.int32, device=dev)
         self.cell_of = torch.zeros(max(N, 1), **u32)
@@ -95,8 +95,8 @@ class Collide:
 
     def exchange_update(self):
         if self.world > 1 and self.exchange:
-            for t in (self.Pm, self.Vm, self.near):
-                allgather_block(t, self.N, self.per, self.rank, self.world, self.group)
+            for b in (self._Pm, self._Vm, self._near):
+                b.gather()
 
     def merge(self, stream=None):
         """Step (2): one virtual merge() per owned active body."""
@@ -105,7 +105,7 @@ class Collide:
 
     def exchange_merge(self):
         if self.world > 1 and self.exchange:
-            allgather_block(self.P, self.N, self.per, self.rank, self.world, self.group)
+            self._P.gather()
 
     def step(self, stream=None):
         self.update(stream)

@@ -83,6 +83,7 @@ struct App {
   static constexpr int kUnroll = 2;
   static constexpr int kUnrollSorted = 2;
   static constexpr int kPrefetch = 2;
+  static constexpr bool kLean = true;  // default launch configuration only (knob sweeps: micro)
   using Base = Cell;
   template <int K>
   using Type = typename TypeOf<K>::T;
@@ -124,10 +125,12 @@ __global__ void k_gen_swap(uint64_t n, const uint8_t* __restrict__ prev, const u
   }
 }
 
-// Fused generation (vf_gen_step): neighbours -> virtual next() -> swap per cell.
+// Fused generation (vf_gen_step / vf_gen_step_rows): neighbours -> virtual
+// next() -> swap per cell, over the cells [off, off + n) of a row slab.
 struct Step {
   uint32_t W, H;
   int torus;
+  uint32_t off;  // first cell of the slab (row0 * W)
   const uint8_t* prev;
   const uint8_t* next;
   uint8_t* nbr;
@@ -135,9 +138,13 @@ struct Step {
   const uint64_t* dead;
   const uint64_t* alive;
   const uint64_t* dying;
-  __device__ __forceinline__ void pre(uint64_t c) const { nbr[c] = count_live(W, H, torus, prev, c); }
-  __device__ __forceinline__ uint64_t ptr(uint64_t c) const { return grid[c]; }
-  __device__ __forceinline__ void post(uint64_t c) const {
+  __device__ __forceinline__ void pre(uint64_t i) const {
+    const uint32_t c = off + (uint32_t)i;
+    nbr[c] = count_live(W, H, torus, prev, c);
+  }
+  __device__ __forceinline__ uint64_t ptr(uint64_t i) const { return grid[off + (uint32_t)i]; }
+  __device__ __forceinline__ void post(uint64_t i) const {
+    const uint32_t c = off + (uint32_t)i;
     const uint8_t s = next[c];
     const int k = kind(s);
     if (k != kind(prev[c])) {
@@ -152,14 +159,15 @@ struct Step {
 
 }  // namespace gen
 
-cudaError_t gen_step(int variant, uint32_t W, uint32_t H, int torus, const uint8_t* prev, uint8_t* next, uint8_t* nbr,
-                     uint64_t* grid, const uint64_t* dead, const uint64_t* alive, const uint64_t* dying,
-                     uint32_t born, uint32_t survive, uint32_t C, const DevTable& tbl, cudaStream_t s) {
+cudaError_t gen_step(int variant, uint32_t W, uint32_t H, int torus, uint32_t row0, uint32_t nrows,
+                     const uint8_t* prev, uint8_t* next, uint8_t* nbr, uint64_t* grid, const uint64_t* dead,
+                     const uint64_t* alive, const uint64_t* dying, uint32_t born, uint32_t survive, uint32_t C,
+                     const DevTable& tbl, cudaStream_t s) {
   vf_gen_next_args a{nbr, next, born, survive, C};
   ArgBlob blob{};
   memcpy(blob.b, &a, sizeof a);
-  const gen::Step st{W, H, torus, prev, next, nbr, grid, dead, alive, dying};
-  return launch_step<gen::App, VF_GEN_NEXT>(variant, (uint64_t)W * H, blob, tbl, st, s);
+  const gen::Step st{W, H, torus, row0 * W, prev, next, nbr, grid, dead, alive, dying};
+  return launch_step<gen::App, VF_GEN_NEXT>(variant, (uint64_t)W * nrows, blob, tbl, st, s);
 }
 
 static const uint32_t kGenBytes[3] = {16, 16, 16};

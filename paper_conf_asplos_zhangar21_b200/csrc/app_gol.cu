@@ -64,6 +64,7 @@ struct App {
   static constexpr int kUnroll = 1;
   static constexpr int kUnrollSorted = 2;
   static constexpr int kPrefetch = 0;
+  static constexpr bool kLean = true;  // default launch configuration only (knob sweeps: micro)
   using Base = Cell;
   template <int K>
   using Type = typename TypeOf<K>::T;
@@ -149,8 +150,9 @@ struct Step {
 // ---------------------------------------------------------------------------
 __device__ __forceinline__ uint8_t ldcg_u8(const uint8_t* p) { return __ldcg(p); }
 
-__device__ __forceinline__ uint8_t count_live_cg(uint32_t W, uint32_t H, int torus, const uint8_t* st, uint64_t c) {
-  const int y = (int)(c / W), x = (int)(c % W);
+__device__ __forceinline__ uint8_t count_live_cg(uint32_t W, uint32_t H, int torus, const uint8_t* st, uint32_t c) {
+  const uint32_t yq = c / W;  // 32-bit (W*H < 2^32): no u64 division subroutine
+  const int y = (int)yq, x = (int)(c - yq * W);
   int n = 0;
 #pragma unroll
   for (int dy = -1; dy <= 1; ++dy)

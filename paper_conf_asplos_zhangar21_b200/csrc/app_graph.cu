@@ -31,6 +31,7 @@ struct Vertex {
   __device__ virtual void cc_update(vf_graph_cc_args a, uint64_t i) = 0;
   __device__ virtual void pr_contrib(vf_graph_pr_args a, uint64_t i) = 0;
   __device__ virtual void pr_update(vf_graph_pr_args a, uint64_t i) = 0;
+  __device__ virtual void bfs_probe_bits(vf_graph_bfs_bits_args a, uint64_t i) = 0;
   uint32_t vid;
   uint32_t deg;
 };
@@ -53,6 +54,21 @@ struct VertexK final : Vertex {
     for (uint64_t k = w.b; k < w.e; ++k) {
       if (a.depth_dev[__ldg(a.col_dev + k)] == a.level) {
         if (atomicCAS(a.depth_dev + vid, -1, a.level + 1) == -1) *(volatile uint32_t*)a.next_count_dev = 1u;
+        return;
+      }
+    }
+  }
+  // bottom-up step over a frontier bitmap (multi-GPU exchange unit)
+  __device__ void bfs_probe_bits(vf_graph_bfs_bits_args a, uint64_t i) {
+    if (*(volatile int32_t*)(a.depth_dev + vid) != -1) return;
+    const Work w = work_of(a.offs_dev, a.chunk_dev, i, vid, deg, a.C);
+    for (uint64_t k = w.b; k < w.e; ++k) {
+      const uint32_t u = __ldg(a.col_dev + k);
+      if ((__ldg(a.frontier_dev + (u >> 5)) >> (u & 31u)) & 1u) {
+        if (atomicCAS(a.depth_dev + vid, -1, a.level + 1) == -1) {
+          atomicOr(a.next_dev + (vid >> 5), 1u << (vid & 31u));
+          *(volatile uint32_t*)a.next_count_dev = 1u;
+        }
         return;
       }
     }
@@ -134,11 +150,12 @@ struct VertexK final : Vertex {
 
 struct App {
   static constexpr int kTypes = 4;
-  static constexpr int kMethods = 5;
+  static constexpr int kMethods = 6;
   static constexpr int kUnroll = 2;
   static constexpr int kUnrollSorted = 2;
   static constexpr int kPrefetch = 2;
-  static constexpr uint32_t kHeavyMask = 0x1Fu;  // one tile per CTA (dispatch.cuh grid_cap)
+  static constexpr bool kLean = true;  // default launch configuration only (knob sweeps: micro)
+  static constexpr uint32_t kHeavyMask = 0x3Fu;  // one tile per CTA (dispatch.cuh grid_cap)
   static constexpr int kMinBlocks = 4;           // <= 64 registers: random gathers need resident warps
   using Base = Vertex;
   template <int K>
@@ -150,7 +167,8 @@ struct App {
     else if constexpr (M == VF_GRAPH_BFS_PROBE) o->bfs_probe(blob_as<vf_graph_bfs_args>(b), i);
     else if constexpr (M == VF_GRAPH_CC_UPDATE) o->cc_update(blob_as<vf_graph_cc_args>(b), i);
     else if constexpr (M == VF_GRAPH_PR_CONTRIB) o->pr_contrib(blob_as<vf_graph_pr_args>(b), i);
-    else o->pr_update(blob_as<vf_graph_pr_args>(b), i);
+    else if constexpr (M == VF_GRAPH_PR_UPDATE) o->pr_update(blob_as<vf_graph_pr_args>(b), i);
+    else o->bfs_probe_bits(blob_as<vf_graph_bfs_bits_args>(b), i);
   }
   template <int M, int K>
   __device__ __forceinline__ static void dcall(Type<K>* o, uint64_t i, const ArgBlob& b) {
@@ -158,7 +176,8 @@ struct App {
     else if constexpr (M == VF_GRAPH_BFS_PROBE) o->Type<K>::bfs_probe(blob_as<vf_graph_bfs_args>(b), i);
     else if constexpr (M == VF_GRAPH_CC_UPDATE) o->Type<K>::cc_update(blob_as<vf_graph_cc_args>(b), i);
     else if constexpr (M == VF_GRAPH_PR_CONTRIB) o->Type<K>::pr_contrib(blob_as<vf_graph_pr_args>(b), i);
-    else o->Type<K>::pr_update(blob_as<vf_graph_pr_args>(b), i);
+    else if constexpr (M == VF_GRAPH_PR_UPDATE) o->Type<K>::pr_update(blob_as<vf_graph_pr_args>(b), i);
+    else o->Type<K>::bfs_probe_bits(blob_as<vf_graph_bfs_bits_args>(b), i);
   }
   __device__ static void construct(uint32_t t, void* mem, const void* arg) {
     construct_switch<App>(t, mem, arg);
@@ -192,9 +211,9 @@ __global__ void k_fill_f32(uint64_t V, float* x, float val) {
 }  // namespace graph
 
 static const uint32_t kGraphBytes[4] = {16, 16, 16, 16};
-static const uint32_t kGraphArgs[5] = {sizeof(vf_graph_bfs_args), sizeof(vf_graph_bfs_args),
+static const uint32_t kGraphArgs[6] = {sizeof(vf_graph_bfs_args), sizeof(vf_graph_bfs_args),
                                        sizeof(vf_graph_cc_args), sizeof(vf_graph_pr_args),
-                                       sizeof(vf_graph_pr_args)};
+                                       sizeof(vf_graph_pr_args), sizeof(vf_graph_bfs_bits_args)};
 
 const AppOps* app_graph() {
   static const AppOps ops = make_ops<graph::App>("graph", kGraphBytes, kGraphArgs);

@@ -134,6 +134,7 @@ struct App {
   static constexpr int kUnroll = 2;
   static constexpr int kUnrollSorted = 2;
   static constexpr int kPrefetch = 2;
+  static constexpr bool kLean = true;  // default launch configuration only (knob sweeps: micro)
   using Base = Element;
   template <int K>
   using Type = typename TypeOf<K>::T;

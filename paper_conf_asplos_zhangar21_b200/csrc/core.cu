@@ -130,6 +130,11 @@ struct vf_ctx {
   std::vector<HeapBatch> heap;
   std::vector<uint64_t> type_count[VF_APP_COUNT];  // live objects per (app, type)
   size_t gran = 2u << 20;
+  // range tables replaced by a rebuild; freed only when no kernel can still
+  // read them (vf_reset / vf_destroy, or after a device sync when many pile up)
+  std::vector<void*> retired;
+  // cuda_packed slabs (vf_alloc_packed), freed at vf_reset
+  std::vector<void*> packed;
   // vf_dispatch_host: copy stream + one event per chunk (created on first use)
   cudaStream_t copy_stream = nullptr;
   std::vector<cudaEvent_t> chunk_events;
@@ -250,10 +255,20 @@ vf_status new_region(vf_ctx* c, Arena& a) {
   return VF_OK;
 }
 
-// Reserve `count` consecutive-in-allocation-order slots of (app,type);
-// appends their addresses to out.
-vf_status alloc_slots(vf_ctx* c, uint32_t app, uint32_t type, uint64_t count,
-                      std::vector<uint64_t>& out) {
+const uint64_t kTagMask = ~((1ull << VF_VA_BITS) - 1);
+
+vf_status tag_check(vf_ctx* c, uint64_t addr) {
+  if (addr & kTagMask)
+    return fail(c, VF_ERR_TAG_BITS, "address 0x%llx uses bits 63:%u (TypePointer needs them 0)",
+                (unsigned long long)addr, VF_VA_BITS);
+  return VF_OK;
+}
+
+// Reserve `count` consecutive-in-allocation-order slots of (app,type); appends
+// their runs as segments (first rank, first address) to `out`, ranks counted
+// from `rank0`.
+vf_status alloc_segments(vf_ctx* c, uint32_t app, uint32_t type, uint64_t count, uint64_t rank0,
+                         std::vector<PlaceSeg>& out) {
   const AppOps* ops = app_ops(app);
   Arena& a = c->arenas[{app, type}];
   if (a.obj_bytes == 0) {
@@ -261,7 +276,6 @@ vf_status alloc_slots(vf_ctx* c, uint32_t app, uint32_t type, uint64_t count,
     a.type = type;
     a.obj_bytes = ops->obj_bytes[type];
   }
-  out.reserve(out.size() + count);
   while (count > 0) {
     if (a.cur < 0 || c->regions[a.cur].used_objs == c->regions[a.cur].cap_objs) {
       vf_status s = new_region(c, a);
@@ -269,8 +283,13 @@ vf_status alloc_slots(vf_ctx* c, uint32_t app, uint32_t type, uint64_t count,
     }
     vf_region& r = c->regions[a.cur];
     const uint64_t take = std::min(count, r.cap_objs - r.used_objs);
-    for (uint64_t k = 0; k < take; ++k) out.push_back(r.start + (r.used_objs + k) * r.obj_bytes);
+    const uint64_t first = r.start + r.used_objs * r.obj_bytes;
+    vf_status s = tag_check(c, first);
+    if (!s) s = tag_check(c, first + take * r.obj_bytes - 1);
+    if (s) return s;
+    out.push_back(PlaceSeg{rank0, first, r.obj_bytes});
     r.used_objs += take;
+    rank0 += take;
     count -= take;
   }
   return VF_OK;
@@ -291,7 +310,7 @@ vf_status ensure_vptrs(vf_ctx* c, uint32_t app) {
 
 // Fig. 3 / P:987-991: sort the app's regions by start, merge exactly-adjacent
 // regions of the same type, upload the table for COAL.
-vf_status rebuild_table(vf_ctx* c, uint32_t app) {
+vf_status rebuild_table(vf_ctx* c, uint32_t app, cudaStream_t stream) {
   vf_status s = ensure_vptrs(c, app);
   if (s) return s;
   AppTable& t = c->tables[app];
@@ -312,26 +331,38 @@ vf_status rebuild_table(vf_ctx* c, uint32_t app) {
   t.K = (uint32_t)t.rows.size();
   t.P = 1;
   while (t.P < t.K) t.P *= 2;
-  if (t.K > t.d_cap) {
-    cudaFree(t.d_start);
-    cudaFree(t.d_end);
-    cudaFree(t.d_type);
-    t.d_cap = std::max<uint32_t>(t.K, 64);
-    CUDA_TRY(c, cudaMalloc(&t.d_start, 8ull * t.d_cap));
-    CUDA_TRY(c, cudaMalloc(&t.d_end, 8ull * t.d_cap));
-    CUDA_TRY(c, cudaMalloc(&t.d_type, 4ull * t.d_cap));
+  // Versioned device table: a new upload never overwrites rows a COAL kernel
+  // still running on another stream may be reading; the old version is
+  // retired and freed once the device is known idle. Uploaded on `stream`.
+  if (t.d_start) {
+    c->retired.push_back(t.d_start);
+    t.d_start = t.d_end = nullptr;
+    t.d_type = nullptr;
   }
   if (t.K) {
-    std::vector<uint64_t> hs(t.K), he(t.K);
-    std::vector<uint32_t> ht(t.K);
+    const size_t bytes = 20ull * t.K;
+    std::vector<unsigned char> host(bytes);
+    uint64_t* hs = reinterpret_cast<uint64_t*>(host.data());
+    uint64_t* he = hs + t.K;
+    uint32_t* ht = reinterpret_cast<uint32_t*>(he + t.K);
     for (uint32_t j = 0; j < t.K; ++j) {
       hs[j] = t.rows[j].start;
       he[j] = t.rows[j].end;
       ht[j] = t.rows[j].type_id;
     }
-    CUDA_TRY(c, cudaMemcpy(t.d_start, hs.data(), 8ull * t.K, cudaMemcpyHostToDevice));
-    CUDA_TRY(c, cudaMemcpy(t.d_end, he.data(), 8ull * t.K, cudaMemcpyHostToDevice));
-    CUDA_TRY(c, cudaMemcpy(t.d_type, ht.data(), 4ull * t.K, cudaMemcpyHostToDevice));
+    void* d = nullptr;
+    CUDA_TRY(c, cudaMalloc(&d, bytes));
+    t.d_start = static_cast<uint64_t*>(d);
+    t.d_end = t.d_start + t.K;
+    t.d_type = reinterpret_cast<uint32_t*>(t.d_end + t.K);
+    CUDA_TRY(c, cudaMemcpyAsync(d, host.data(), bytes, cudaMemcpyHostToDevice, stream));
+    CUDA_TRY(c, cudaStreamSynchronize(stream));  // `host` goes out of scope
+  }
+  t.d_cap = t.K;
+  if (c->retired.size() > 64) {
+    CUDA_TRY(c, cudaDeviceSynchronize());
+    for (void* p : c->retired) cudaFree(p);
+    c->retired.clear();
   }
   c->all_rows.clear();
   for (uint32_t a = 0; a < VF_APP_COUNT; ++a)
@@ -359,15 +390,6 @@ DevTable dev_table(vf_ctx* c, uint32_t app) {
 vf_status check_app(vf_ctx* c, uint32_t app) {
   if (!c) return VF_ERR_INVALID;
   if (!app_ops(app)) return fail(c, VF_ERR_INVALID, "unknown app %u", app);
-  return VF_OK;
-}
-
-const uint64_t kTagMask = ~((1ull << VF_VA_BITS) - 1);
-
-vf_status tag_check(vf_ctx* c, uint64_t addr) {
-  if (addr & kTagMask)
-    return fail(c, VF_ERR_TAG_BITS, "address 0x%llx uses bits 63:%u (TypePointer needs them 0)",
-                (unsigned long long)addr, VF_VA_BITS);
   return VF_OK;
 }
 
@@ -504,6 +526,10 @@ vf_status vf_reset(vf_ctx* c) {
     cudaFree(h.d_ptrs);
   }
   c->heap.clear();
+  for (void* p : c->retired) cudaFree(p);
+  c->retired.clear();
+  for (void* p : c->packed) cudaFree(p);
+  c->packed.clear();
   for (size_t r = 0; r < c->region_malloc.size(); ++r)
     if (c->region_malloc[r]) cudaFree(c->region_malloc[r]);
   Drv& d = drv();
@@ -537,11 +563,10 @@ void vf_destroy(vf_ctx* c) {
   for (auto& kv : c->arenas)
     if (kv.second.va) d.addr_free(kv.second.va, kv.second.va_size);
   for (AppTable& t : c->tables) {
-    cudaFree(t.d_start);
-    cudaFree(t.d_end);
-    cudaFree(t.d_type);
+    cudaFree(t.d_start);  // one allocation holds start, end and type
     cudaFree(t.d_vptr);
   }
+  for (void* p : c->retired) cudaFree(p);
   for (cudaEvent_t e : c->chunk_events) cudaEventDestroy(e);
   if (c->copy_stream) cudaStreamDestroy(c->copy_stream);
   delete c;
@@ -556,41 +581,53 @@ vf_status vf_alloc_typed_batch(vf_ctx* c, uint32_t app, const uint32_t* type_ids
   if (!type_ids_dev || !out_ptrs_dev) return fail(c, VF_ERR_INVALID, "null device pointer");
   if ((st = set_device(c))) return st;
   const AppOps* ops = app_ops(app);
-  std::vector<uint32_t> types(count);
-  CUDA_TRY(c, cudaMemcpyAsync(types.data(), type_ids_dev, 4ull * count, cudaMemcpyDeviceToHost, S(stream)));
-  CUDA_TRY(c, cudaStreamSynchronize(S(stream)));
-  std::vector<uint64_t> cnt(ops->ntypes, 0);
-  for (uint64_t i = 0; i < count; ++i) {
-    if (types[i] >= ops->ntypes)
-      return fail(c, VF_ERR_INVALID, "type id %u at %llu >= ntypes %u", types[i],
-                  (unsigned long long)i, ops->ntypes);
-    ++cnt[types[i]];
-  }
+  if (ops->ntypes > 32) return fail(c, VF_ERR_TOO_MANY_TYPES, "device ranking handles <= 32 types");
+  cudaStream_t s = S(stream);
+  // (1) per-type exclusive prefix counts on the device (alloc.cu); only the
+  // T totals come back to the host, which sizes and maps the regions
+  const uint64_t nch = rank_chunks(count);
+  unsigned char* scratch = nullptr;
+  const size_t hist_bytes = 128ull * nch;
+  CUDA_TRY(c, cudaMallocAsync(reinterpret_cast<void**>(&scratch), hist_bytes + 8 * 32 + 16, s));
+  uint32_t* hist = reinterpret_cast<uint32_t*>(scratch);
+  unsigned long long* totals = reinterpret_cast<unsigned long long*>(scratch + hist_bytes);
+  uint32_t* bad = reinterpret_cast<uint32_t*>(scratch + hist_bytes + 8 * 32);
+  struct Guard {
+    unsigned char* p;
+    cudaStream_t s;
+    ~Guard() { cudaFreeAsync(p, s); }
+  } guard{scratch, s};
+  CUDA_TRY(c, cudaMemsetAsync(bad, 0, 4, s));
+  CUDA_TRY(c, rank_hist(type_ids_dev, count, ops->ntypes, hist, bad, totals, s));
+  unsigned long long h_tot[32] = {0};
+  uint32_t h_bad = 0;
+  CUDA_TRY(c, cudaMemcpyAsync(h_tot, totals, 8ull * ops->ntypes, cudaMemcpyDeviceToHost, s));
+  CUDA_TRY(c, cudaMemcpyAsync(&h_bad, bad, 4, cudaMemcpyDeviceToHost, s));
+  CUDA_TRY(c, cudaStreamSynchronize(s));
+  if (h_bad) return fail(c, VF_ERR_INVALID, "a type id >= ntypes %u", ops->ntypes);
   if (tag && ops->ntypes > 127) return fail(c, VF_ERR_TOO_MANY_TYPES, "7-bit tag holds 127 types");
-  std::vector<std::vector<uint64_t>> slots(ops->ntypes);
-  for (uint32_t t = 0; t < ops->ntypes; ++t)
-    if (cnt[t] && (st = alloc_slots(c, app, t, cnt[t], slots[t]))) return st;
-  c->type_count[app].resize(ops->ntypes, 0);
-  for (uint32_t t = 0; t < ops->ntypes; ++t) c->type_count[app][t] += cnt[t];
-  std::vector<uint64_t> ptrs(count);
-  std::vector<uint64_t> rank(ops->ntypes, 0);
-  for (uint64_t i = 0; i < count; ++i) {
-    const uint32_t t = types[i];
-    const uint64_t a = slots[t][rank[t]++];
-    ptrs[i] = a;
-  }
+  // (2) regions: each type's slots as segments (rank range -> first address)
+  std::vector<PlaceSeg> segs;
+  std::vector<uint32_t> first(ops->ntypes + 1, 0);
   for (uint32_t t = 0; t < ops->ntypes; ++t) {
-    if (!slots[t].empty()) {
-      if ((st = tag_check(c, slots[t].front()))) return st;
-      if ((st = tag_check(c, slots[t].back() + ops->obj_bytes[t] - 1))) return st;
-    }
+    first[t] = (uint32_t)segs.size();
+    if (h_tot[t] && (st = alloc_segments(c, app, t, h_tot[t], 0, segs))) return st;
   }
-  if (tag)
-    for (uint64_t i = 0; i < count; ++i) ptrs[i] = tag_ptr(ptrs[i], types[i]);
-  CUDA_TRY(c, cudaMemcpyAsync(out_ptrs_dev, ptrs.data(), 8ull * count, cudaMemcpyHostToDevice, S(stream)));
-  CUDA_TRY(c, ops->construct(type_ids_dev, out_ptrs_dev, ctor_args_dev, ctor_arg_bytes, count, S(stream)));
-  CUDA_TRY(c, cudaStreamSynchronize(S(stream)));
-  return rebuild_table(c, app);
+  first[ops->ntypes] = (uint32_t)segs.size();
+  c->type_count[app].resize(ops->ntypes, 0);
+  for (uint32_t t = 0; t < ops->ntypes; ++t) c->type_count[app][t] += h_tot[t];
+  // (3) place every object at its slot (device), then construct it there
+  const size_t seg_bytes = sizeof(PlaceSeg) * segs.size(), first_bytes = 4ull * first.size();
+  unsigned char* d_seg = nullptr;
+  CUDA_TRY(c, cudaMallocAsync(reinterpret_cast<void**>(&d_seg), seg_bytes + first_bytes, s));
+  Guard guard2{d_seg, s};
+  CUDA_TRY(c, cudaMemcpyAsync(d_seg, segs.data(), seg_bytes, cudaMemcpyHostToDevice, s));
+  CUDA_TRY(c, cudaMemcpyAsync(d_seg + seg_bytes, first.data(), first_bytes, cudaMemcpyHostToDevice, s));
+  CUDA_TRY(c, rank_place(type_ids_dev, count, hist, reinterpret_cast<const PlaceSeg*>(d_seg),
+                         reinterpret_cast<const uint32_t*>(d_seg + seg_bytes), tag, out_ptrs_dev, s));
+  CUDA_TRY(c, ops->construct(type_ids_dev, out_ptrs_dev, ctor_args_dev, ctor_arg_bytes, count, s));
+  CUDA_TRY(c, cudaStreamSynchronize(s));
+  return rebuild_table(c, app, s);
 }
 
 vf_status vf_alloc_typed(vf_ctx* c, uint32_t app, uint32_t type_id, uint64_t count,
@@ -603,8 +640,7 @@ vf_status vf_alloc_typed(vf_ctx* c, uint32_t app, uint32_t type_id, uint64_t cou
   if ((st = set_device(c))) return st;
   uint32_t* d_types = nullptr;
   CUDA_TRY(c, cudaMallocAsync(&d_types, 4ull * count, S(stream)));
-  std::vector<uint32_t> h(count, type_id);
-  cudaError_t e = cudaMemcpyAsync(d_types, h.data(), 4ull * count, cudaMemcpyHostToDevice, S(stream));
+  cudaError_t e = fill_u32(d_types, count, type_id, S(stream));
   if (e == cudaSuccess)
     st = vf_alloc_typed_batch(c, app, d_types, count, ctor_args_dev, ctor_arg_bytes, out_ptrs_dev,
                               tag, stream);
@@ -612,6 +648,35 @@ vf_status vf_alloc_typed(vf_ctx* c, uint32_t app, uint32_t type_id, uint64_t cou
   cudaStreamSynchronize(S(stream));
   if (e != cudaSuccess) return fail(c, VF_ERR_CUDA, "%s", cudaGetErrorString(e));
   return st;
+}
+
+vf_status vf_alloc_packed(vf_ctx* c, uint32_t app, const uint32_t* type_ids_dev, uint64_t count,
+                          const void* ctor_args_dev, uint32_t ctor_arg_bytes, uint64_t* out_ptrs_dev,
+                          void* stream) {
+  vf_status st = check_app(c, app);
+  if (st) return st;
+  if (count == 0) return VF_OK;
+  if (!type_ids_dev || !out_ptrs_dev) return fail(c, VF_ERR_INVALID, "null device pointer");
+  if ((st = set_device(c))) return st;
+  const AppOps* ops = app_ops(app);
+  uint64_t stride = 0;
+  for (uint32_t t = 0; t < ops->ntypes; ++t) stride = std::max<uint64_t>(stride, ops->obj_bytes[t]);
+  stride = (stride + 15) & ~15ull;
+  void* slab = nullptr;
+  cudaError_t e = cudaMalloc(&slab, stride * count);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    return fail(c, VF_ERR_OOM, "cudaMalloc(%llu) for a packed slab: %s",
+                (unsigned long long)(stride * count), cudaGetErrorString(e));
+  }
+  c->packed.push_back(slab);
+  cudaStream_t s = S(stream);
+  CUDA_TRY(c, place_packed(reinterpret_cast<uint64_t>(slab), stride, count, out_ptrs_dev, s));
+  CUDA_TRY(c, ops->construct(type_ids_dev, out_ptrs_dev, ctor_args_dev, ctor_arg_bytes, count, s));
+  CUDA_TRY(c, cudaStreamSynchronize(s));
+  c->type_count[app].resize(ops->ntypes, 0);
+  c->type_count[app][0] += count;  // types unknown on the host: marks the app live (launch heuristics)
+  return ensure_vptrs(c, app);
 }
 
 vf_status vf_alloc_cuda(vf_ctx* c, uint32_t app, const uint32_t* type_ids_dev, uint64_t count,
@@ -791,6 +856,7 @@ vf_status vf_gol_step(vf_ctx* c, vf_variant v, uint32_t W, uint32_t H, int torus
   vf_status st = check_app(c, VF_APP_GOL);
   if (st) return st;
   if ((unsigned)v > VF_TYPEPTR) return fail(c, VF_ERR_INVALID, "variant %d", (int)v);
+  if ((uint64_t)W * H > 0xFFFFFFFFull) return fail(c, VF_ERR_INVALID, "W*H > 2^32-1 cells");
   if ((uint64_t)W * H && (!prev_dev || !next_dev || !nbr_dev || !grid_dev || !alive_dev || !dead_dev))
     return fail(c, VF_ERR_INVALID, "gol_step arguments");
   if ((st = set_device(c)) || (st = ensure_vptrs(c, VF_APP_GOL))) return st;
@@ -807,6 +873,7 @@ vf_status vf_gol_run(vf_ctx* c, vf_variant v, uint32_t W, uint32_t H, int torus,
   vf_status st = check_app(c, VF_APP_GOL);
   if (st) return st;
   if ((unsigned)v > VF_TYPEPTR) return fail(c, VF_ERR_INVALID, "variant %d", (int)v);
+  if ((uint64_t)W * H > 0xFFFFFFFFull) return fail(c, VF_ERR_INVALID, "W*H > 2^32-1 cells");
   if ((uint64_t)W * H && gens &&
       (!state0_dev || !state1_dev || !nbr_dev || !grid_dev || !alive_dev || !dead_dev || !barrier_dev))
     return fail(c, VF_ERR_INVALID, "gol_run arguments");
@@ -818,22 +885,35 @@ vf_status vf_gol_run(vf_ctx* c, vf_variant v, uint32_t W, uint32_t H, int torus,
   return VF_OK;
 }
 
-vf_status vf_gen_step(vf_ctx* c, vf_variant v, uint32_t W, uint32_t H, int torus, const uint8_t* prev_dev,
-                      uint8_t* next_dev, uint8_t* nbr_dev, uint64_t* grid_dev, const uint64_t* dead_dev,
-                      const uint64_t* alive_dev, const uint64_t* dying_dev, uint32_t born_mask,
-                      uint32_t survive_mask, uint32_t C, void* stream) {
+vf_status vf_gen_step_rows(vf_ctx* c, vf_variant v, uint32_t W, uint32_t H, int torus, uint32_t row0,
+                           uint32_t nrows, const uint8_t* prev_dev, uint8_t* next_dev, uint8_t* nbr_dev,
+                           uint64_t* grid_dev, const uint64_t* dead_dev, const uint64_t* alive_dev,
+                           const uint64_t* dying_dev, uint32_t born_mask, uint32_t survive_mask, uint32_t C,
+                           void* stream) {
   vf_status st = check_app(c, VF_APP_GEN);
   if (st) return st;
   if ((unsigned)v > VF_TYPEPTR) return fail(c, VF_ERR_INVALID, "variant %d", (int)v);
-  if ((uint64_t)W * H && (!prev_dev || !next_dev || !nbr_dev || !grid_dev || !dead_dev || !alive_dev || !dying_dev))
+  if ((uint64_t)W * H > 0xFFFFFFFFull) return fail(c, VF_ERR_INVALID, "W*H = %llu > 2^32-1 cells",
+                                                  (unsigned long long)W * H);
+  if ((uint64_t)row0 + nrows > H) return fail(c, VF_ERR_INVALID, "rows [%u, %u) outside H = %u", row0, row0 + nrows, H);
+  if ((uint64_t)W * nrows && (!prev_dev || !next_dev || !nbr_dev || !grid_dev || !dead_dev || !alive_dev || !dying_dev))
     return fail(c, VF_ERR_INVALID, "gen_step arguments");
   if (C < 2 || C > 255) return fail(c, VF_ERR_INVALID, "C = %u", C);
   if ((st = set_device(c)) || (st = ensure_vptrs(c, VF_APP_GEN))) return st;
   if (v == VF_COAL && c->tables[VF_APP_GEN].K > VF_MAX_RANGES)
     return fail(c, VF_ERR_TABLE_FULL, "K = %u > %u", c->tables[VF_APP_GEN].K, VF_MAX_RANGES);
-  CUDA_TRY(c, gen_step((int)v, W, H, torus, prev_dev, next_dev, nbr_dev, grid_dev, dead_dev, alive_dev, dying_dev,
-                       born_mask, survive_mask, C, dev_table(c, VF_APP_GEN), reinterpret_cast<cudaStream_t>(stream)));
+  CUDA_TRY(c, gen_step((int)v, W, H, torus, row0, nrows, prev_dev, next_dev, nbr_dev, grid_dev, dead_dev, alive_dev,
+                       dying_dev, born_mask, survive_mask, C, dev_table(c, VF_APP_GEN),
+                       reinterpret_cast<cudaStream_t>(stream)));
   return VF_OK;
+}
+
+vf_status vf_gen_step(vf_ctx* c, vf_variant v, uint32_t W, uint32_t H, int torus, const uint8_t* prev_dev,
+                      uint8_t* next_dev, uint8_t* nbr_dev, uint64_t* grid_dev, const uint64_t* dead_dev,
+                      const uint64_t* alive_dev, const uint64_t* dying_dev, uint32_t born_mask,
+                      uint32_t survive_mask, uint32_t C, void* stream) {
+  return vf_gen_step_rows(c, v, W, H, torus, 0, H, prev_dev, next_dev, nbr_dev, grid_dev, dead_dev, alive_dev,
+                          dying_dev, born_mask, survive_mask, C, stream);
 }
 
 vf_status vf_dispatch_cuda(vf_ctx* c, uint32_t app, uint32_t m, const uint64_t* o, uint64_t n,

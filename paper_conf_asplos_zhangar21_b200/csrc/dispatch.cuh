@@ -20,6 +20,7 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <mutex>
 #include <new>
 #include <type_traits>
 #include <utility>
@@ -120,7 +121,8 @@ struct ResolveCOAL {
     const uint64_t* s_start = reinterpret_cast<const uint64_t*>(smem);
     const uint64_t* s_end = s_start + P;
     const uint32_t* s_type = reinterpret_cast<const uint32_t*>(s_end + P);
-    a = p;
+    a = strip(p);  // a TypePointer-tagged pointer is searched (and dereferenced) by its address
+    p = a;
     (void)hint;
     uint32_t j = 0;
     for (uint32_t step = P >> 1; step > 0; step >>= 1) {
@@ -346,13 +348,15 @@ __global__ void __launch_bounds__(kBlock, 4) k_dispatch_pipe(const uint64_t* __r
   const uint64_t full = n / WT;
   const uint64_t gw = (uint64_t)blockIdx.x * L::kWarps + warp;
   const uint64_t nw = (uint64_t)gridDim.x * L::kWarps;
-  const uint64_t mine = gw < full ? (full - 1 - gw) / nw + 1 : 0;
+  // warp tile k of this warp is tile gw + k*nw; it exists iff that is < full
+  // (a multiply instead of a 64-bit division: no CALL into the u64 divide)
+  auto has = [&](uint64_t k) { return gw + k * nw < full; };
   auto tile_base = [&](uint64_t k) { return (gw + k * nw) * WT; };
 
   if (lane == 0) {
     for (int s = 0; s < S; ++s) mbar_init(&bars[s], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    for (int s = 0; s < S && (uint64_t)s < mine; ++s) {
+    for (int s = 0; s < S && has((uint64_t)s); ++s) {
       mbar_expect_tx(&bars[s], WT * sizeof(uint64_t));
       tma_load_1d(ring + (size_t)s * WT, objs + tile_base(s), WT * sizeof(uint64_t), &bars[s]);
     }
@@ -370,7 +374,7 @@ __global__ void __launch_bounds__(kBlock, 4) k_dispatch_pipe(const uint64_t* __r
 #pragma unroll
     for (int j = 0; j < U; ++j) p[j] = ring[(size_t)s * WT + j * 32 + lane];
     __syncwarp();  // the whole warp holds its pointers: the stage can be refilled
-    if (lane == 0 && k + S < mine) {
+    if (lane == 0 && has(k + S)) {
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
       mbar_expect_tx(&bars[s], WT * sizeof(uint64_t));
       tma_load_1d(ring + (size_t)s * WT, objs + tile_base(k + S), WT * sizeof(uint64_t), &bars[s]);
@@ -378,13 +382,13 @@ __global__ void __launch_bounds__(kBlock, 4) k_dispatch_pipe(const uint64_t* __r
     resolve_tile<App, M, R, U, PF>(smem, tbl.P, p, a, t, w, hint);
   };
 
-  if (mine > 0) fetch(0, pc, ac, tc, wc);
-  for (uint64_t k = 0; k < mine; ++k) {
+  if (has(0)) fetch(0, pc, ac, tc, wc);
+  for (uint64_t k = 0; has(k); ++k) {
 #pragma unroll
     for (int j = 0; j < U; ++j) sink ^= wc[j];
     uint64_t pn[U], an[U];
     uint32_t tn[U], wn[U];
-    if (k + 1 < mine) fetch(k + 1, pn, an, tn, wn);
+    if (has(k + 1)) fetch(k + 1, pn, an, tn, wn);
     const uint64_t base = tile_base(k);
 #pragma unroll
     for (int j = 0; j < U; ++j) group_call<App, M>(tc[j], ac[j], pc[j], base + j * 32 + lane, args, tbl);
@@ -758,7 +762,7 @@ __device__ __forceinline__ uint32_t resolve_rule(int variant, const unsigned cha
     return kNF;
   }
   // CUDA / SharedOA: the embedded vTable* (Fig. 1a load A), mapped to a type id
-  const uint64_t vp = *reinterpret_cast<const uint64_t*>(p);
+  const uint64_t vp = *reinterpret_cast<const uint64_t*>(strip(p));
   for (uint32_t k = 0; k < tbl.ntypes; ++k)
     if (tbl.vptr[k] == vp) return k;
   return kNF;
@@ -797,15 +801,54 @@ __global__ void k_verify(int variant, const uint64_t* __restrict__ ptrs, uint64_
 // ---------------------------------------------------------------------------
 // Host-side launch helpers shared by the app modules.
 // ---------------------------------------------------------------------------
+// Launch-configuration caches are per device (a second ctx on another GPU
+// gets its own attribute set-up and SM count) and guarded by a mutex (two
+// ctxs may launch from two host threads).
+constexpr int kMaxDevices = 64;
+inline int current_device() {
+  int dev = 0;
+  cudaGetDevice(&dev);
+  return dev & (kMaxDevices - 1);
+}
+inline std::mutex& launch_cache_mutex() {
+  static std::mutex m;
+  return m;
+}
+
 inline int num_sms() {
-  static int sms = 0;
-  if (!sms) {
-    int dev = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    if (sms <= 0) sms = 148;
+  static int sms[kMaxDevices] = {0};
+  const int dev = current_device();
+  if (!sms[dev]) {
+    std::lock_guard<std::mutex> lk(launch_cache_mutex());
+    int v = 0;
+    int d = 0;
+    cudaGetDevice(&d);
+    cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, d);
+    sms[dev] = v > 0 ? v : 148;
   }
-  return sms;
+  return sms[dev];
+}
+
+// Resident CTAs per SM of kernel `Kern` at `smem` dynamic shared memory on the
+// current device (sets the opt-in dynamic smem attribute above 48 KB once per
+// device and size).
+template <auto Kern>
+inline int occupancy(size_t smem, int block = kBlock) {
+  struct Slot {
+    int occ = -1;
+    size_t sm = ~(size_t)0;
+  };
+  static Slot slots[kMaxDevices];
+  Slot& sl = slots[current_device()];
+  std::lock_guard<std::mutex> lk(launch_cache_mutex());
+  if (sl.occ < 0 || sl.sm != smem) {
+    if (smem > 32 * 1024) cudaFuncSetAttribute(Kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    int occ = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, Kern, block, smem);
+    sl.occ = occ < 1 ? 1 : occ;
+    sl.sm = smem;
+  }
+  return sl.occ;
 }
 
 inline size_t table_smem(const DevTable& t) { return table_smem_dev(t.P); }
@@ -840,17 +883,9 @@ inline uint64_t grid_cap(int occ) {
 template <class App, int M, class R, int U, int PF>
 cudaError_t launch_grouped(const uint64_t* objs, uint64_t n, const ArgBlob& args,
                            const DevTable& tbl, cudaStream_t s) {
-  auto kern = k_dispatch_grouped<App, M, R, U, PF>;
+  constexpr auto kern = k_dispatch_grouped<App, M, R, U, PF>;
   const size_t sm = R::kNeedsTable ? table_smem(tbl) : 0;
-  static int occ = -1;
-  static size_t occ_sm = ~(size_t)0;
-  if (occ < 0 || occ_sm != sm) {
-    if (sm > 48 * 1024)
-      cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kBlock, sm);
-    if (occ < 1) occ = 1;
-    occ_sm = sm;
-  }
+  const int occ = occupancy<kern>(sm);
   const unsigned grid = grid_for(n, (uint64_t)kBlock * U, grid_cap<App, M>(occ));
   kern<<<grid, kBlock, sm, s>>>(objs, n, args, tbl);
   note_launch();
@@ -870,17 +905,9 @@ cudaError_t launch_virtual(const uint64_t* objs, uint64_t n, const ArgBlob& args
 template <class App, int M, class R, int U, int PF, int S>
 cudaError_t launch_pipe(const uint64_t* objs, uint64_t n, const ArgBlob& args, const DevTable& tbl,
                         cudaStream_t s) {
-  auto kern = k_dispatch_pipe<App, M, R, U, PF, S>;
+  constexpr auto kern = k_dispatch_pipe<App, M, R, U, PF, S>;
   const size_t sm = PipeSmem<U, S>::bytes(R::kNeedsTable ? table_smem(tbl) : 0);
-  static int occ = -1;
-  static size_t occ_sm = ~(size_t)0;
-  if (occ < 0 || occ_sm != sm) {
-    if (sm > 48 * 1024)
-      cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kBlock, sm);
-    if (occ < 1) occ = 1;
-    occ_sm = sm;
-  }
+  const int occ = occupancy<kern>(sm);
   const uint64_t tiles = n / ((uint64_t)kBlock * U);  // CTA-sized tiles of warp tiles
   const unsigned grid = grid_for(tiles, 1, (uint64_t)num_sms() * occ);
   kern<<<grid, kBlock, sm, s>>>(objs, n, args, tbl);
@@ -891,17 +918,9 @@ cudaError_t launch_pipe(const uint64_t* objs, uint64_t n, const ArgBlob& args, c
 template <class App, int M, class R, int U, int PF>
 cudaError_t launch_sorted(const uint64_t* objs, uint64_t n, const ArgBlob& args, const DevTable& tbl,
                           cudaStream_t s) {
-  auto kern = k_dispatch_sorted<App, M, R, U, PF>;
+  constexpr auto kern = k_dispatch_sorted<App, M, R, U, PF>;
   const size_t sm = SortSmem<U>::bytes(R::kNeedsTable ? table_smem(tbl) : 0);
-  static int occ = -1;
-  static size_t occ_sm = ~(size_t)0;
-  if (occ < 0 || occ_sm != sm) {
-    if (sm > 48 * 1024)
-      cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kBlock, sm);
-    if (occ < 1) occ = 1;
-    occ_sm = sm;
-  }
+  const int occ = occupancy<kern>(sm);
   const unsigned grid = grid_for(n, (uint64_t)kBlock * U, grid_cap<App, M>(occ));
   kern<<<grid, kBlock, sm, s>>>(objs, n, args, tbl);
   note_launch();
@@ -972,16 +991,9 @@ cudaError_t launch_grouped_tuned(const uint64_t* objs, uint64_t n, const ArgBlob
 template <class App, int M, class R>
 cudaError_t launch_indirect(const uint64_t* objs, uint64_t n, const ArgBlob& args, const DevTable& tbl,
                             cudaStream_t s) {
-  auto kern = k_dispatch_indirect<App, M, R>;
+  constexpr auto kern = k_dispatch_indirect<App, M, R>;
   const size_t sm = R::kNeedsTable ? table_smem(tbl) : 0;
-  static int occ = -1;
-  static size_t occ_sm = ~(size_t)0;
-  if (occ < 0 || occ_sm != sm) {
-    if (sm > 40 * 1024) cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kBlock, sm);
-    if (occ < 1) occ = 1;
-    occ_sm = sm;
-  }
+  const int occ = occupancy<kern>(sm);
   kern<<<grid_for(n, kBlock, (uint64_t)num_sms() * occ), kBlock, sm, s>>>(objs, n, args, tbl);
   note_launch();
   return cudaGetLastError();
@@ -1156,16 +1168,9 @@ __global__ void __launch_bounds__(kBlock) k_step_virtual(uint64_t n, ArgBlob arg
 template <class App, int M, class R, class Step>
 cudaError_t launch_step_grouped(uint64_t n, const ArgBlob& args, const DevTable& tbl, const Step& st,
                                 cudaStream_t s) {
-  auto kern = k_step_grouped<App, M, R, Step>;
+  constexpr auto kern = k_step_grouped<App, M, R, Step>;
   const size_t sm = R::kNeedsTable ? table_smem(tbl) : 0;
-  static int occ = -1;
-  static size_t occ_sm = ~(size_t)0;
-  if (occ < 0 || occ_sm != sm) {
-    if (sm > 48 * 1024) cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kBlock, sm);
-    if (occ < 1) occ = 1;
-    occ_sm = sm;
-  }
+  const int occ = occupancy<kern>(sm);
   kern<<<grid_for(n, kBlock, (uint64_t)num_sms() * occ), kBlock, sm, s>>>(n, args, tbl, st);
   note_launch();
   return cudaGetLastError();
@@ -1189,10 +1194,13 @@ cudaError_t launch_step(int variant, uint64_t n, const ArgBlob& args, const DevT
   return cudaErrorInvalidValue;
 }
 
-// live (state == 1) neighbours of cell c of a W x H grid (dead border, or torus)
+// live (state == 1) neighbours of cell c of a W x H grid (dead border, or
+// torus). 32-bit index arithmetic (W*H < 2^32, checked at the ABI): a 64-bit
+// `c / W` compiles to a CALL into the u64 division subroutine.
 __device__ __forceinline__ uint8_t count_live(uint32_t W, uint32_t H, int torus, const uint8_t* __restrict__ st,
-                                              uint64_t c) {
-  const int y = (int)(c / W), x = (int)(c % W);
+                                              uint32_t c) {
+  const uint32_t yq = c / W;
+  const int y = (int)yq, x = (int)(c - yq * W);
   int n = 0;
 #pragma unroll
   for (int dy = -1; dy <= 1; ++dy)
@@ -1206,7 +1214,7 @@ __device__ __forceinline__ uint8_t count_live(uint32_t W, uint32_t H, int torus,
       } else if (yy < 0 || yy >= (int)H || xx < 0 || xx >= (int)W) {
         continue;
       }
-      n += st[(uint64_t)yy * W + xx] == 1;
+      n += st[(uint32_t)yy * W + (uint32_t)xx] == 1;
     }
   return (uint8_t)n;
 }

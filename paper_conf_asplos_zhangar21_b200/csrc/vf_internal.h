@@ -81,9 +81,29 @@ cudaError_t gol_step(int variant, uint32_t W, uint32_t H, int torus, const uint8
 cudaError_t gol_run(int variant, uint32_t W, uint32_t H, int torus, uint8_t* buf0, uint8_t* buf1, uint8_t* nbr,
                     uint64_t* grid, const uint64_t* alive, const uint64_t* dead, uint32_t gens, unsigned* bar,
                     const DevTable& tbl, cudaStream_t s);
-cudaError_t gen_step(int variant, uint32_t W, uint32_t H, int torus, const uint8_t* prev, uint8_t* next, uint8_t* nbr,
-                     uint64_t* grid, const uint64_t* dead, const uint64_t* alive, const uint64_t* dying,
-                     uint32_t born, uint32_t survive, uint32_t C, const DevTable& tbl, cudaStream_t s);
+cudaError_t gen_step(int variant, uint32_t W, uint32_t H, int torus, uint32_t row0, uint32_t nrows,
+                     const uint8_t* prev, uint8_t* next, uint8_t* nbr, uint64_t* grid, const uint64_t* dead,
+                     const uint64_t* alive, const uint64_t* dying, uint32_t born, uint32_t survive, uint32_t C,
+                     const DevTable& tbl, cudaStream_t s);
+
+// Batched typed allocation on the device (alloc.cu). A type's free slots, in
+// allocation order, are a list of segments: ranks [rank0, next segment's
+// rank0) live at addr + (rank - rank0) * obj_bytes.
+struct PlaceSeg {
+  uint64_t rank0;
+  uint64_t addr;
+  uint64_t obj_bytes;
+};
+uint64_t rank_chunks(uint64_t n);  // hist rows (32 u32 each) needed for n objects
+// per-chunk type histogram -> in-place exclusive scan per type; totals[t] =
+// objects of type t; *bad != 0 if a type id >= ntypes (ntypes <= 32)
+cudaError_t rank_hist(const uint32_t* types, uint64_t n, uint32_t ntypes, uint32_t* hist, uint32_t* bad,
+                      unsigned long long* totals, cudaStream_t s);
+// out[i] = slot of object i (its rank among same-type objects of lower index), tagged if tag
+cudaError_t rank_place(const uint32_t* types, uint64_t n, const uint32_t* hist, const PlaceSeg* segs,
+                       const uint32_t* seg_first, int tag, uint64_t* out, cudaStream_t s);
+cudaError_t place_packed(uint64_t base, uint64_t stride, uint64_t n, uint64_t* out, cudaStream_t s);
+cudaError_t fill_u32(uint32_t* x, uint64_t n, uint32_t v, cudaStream_t s);
 
 // Benchmark / ablation knobs set through vf_set_tuning (-1 = app default).
 struct Tuning {

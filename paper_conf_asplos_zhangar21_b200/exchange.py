@@ -1,0 +1,158 @@
+"""Per-step exchange of the multi-GPU apps.
+
+The paper runs on one GPU; the exchange is this build's
+extension for the shardable apps. One process per GPU; every rank owns a
+contiguous block of ids (vertices, bodies, node rows) and the step kernels
+write only owned entries. What the next step needs from other ranks is
+exchanged here, with NO per-call allocation:
+
+* ``BlockArray``: a per-id array that lives in a persistent buffer padded to
+  ``per * world`` rows. ``view`` (the first n rows) is what the kernels index.
+  ``gather()`` is ONE ``all_gather_into_tensor`` whose input is this rank's
+  own block of the same buffer (NCCL in-place all-gather: no copy). The
+  graph's frontier bitmap, CC labels, PR contributions, N-body / STUT
+  positions all use it.
+* ``HaloRows``: the GEN row slabs' halo exchange, ``batch_isend_irecv`` of
+  one boundary row to each neighbour slab per generation.
+* ``allreduce_``: in-place sum (BFS "changed", PR dangling mass).
+
+CPU tests drive the same code over ``gloo`` process groups. gloo cannot move
+CUDA tensors in these collectives, so when the group is gloo and the tensor
+is on a GPU, the owned block is staged through a pinned host buffer (the
+2-process GPU tests run both ranks on one device that way); with NCCL nothing
+is staged.
+"""
+from __future__ import annotations
+
+import torch
+
+
+def _dist():
+    import torch.distributed as dist
+    return dist
+
+
+def block_range(n: int, rank: int, world: int, align: int = 1):
+    """Owned block [lo, hi) of `rank` and the per-rank block size `per`
+    (ceil(n / world) rounded up to `align`, so that bitmap slices are whole words)."""
+    per = -(-n // world) if world > 0 else n
+    per = -(-per // align) * align if align > 1 else per
+    return min(n, rank * per), min(n, (rank + 1) * per), per
+
+
+def _staged(t: torch.Tensor, group) -> bool:
+    return t.is_cuda and _dist().get_backend(group) == "gloo"
+
+
+class BlockArray:
+    """Persistent padded per-id array whose owned blocks are all-gathered in place."""
+
+    def __init__(self, n: int, per: int, rank: int, world: int, dtype, device, rest=(), group=None,
+                 fill=None):
+        self.n, self.per, self.rank, self.world, self.group = n, per, rank, world, group
+        rows = per * world if world > 1 else n
+        self.buf = torch.empty((max(rows, 1),) + tuple(rest), dtype=dtype, device=device)
+        if fill is not None:
+            self.buf.fill_(fill)
+        self.view = self.buf[:n]
+        self.mine = self.buf[rank * per:(rank + 1) * per] if world > 1 else self.view
+        self._host = None
+
+    def data_ptr(self) -> int:
+        return self.view.data_ptr()
+
+    def gather(self):
+        """After the call every rank holds every rank's block (one collective)."""
+        if self.world == 1:
+            return
+        dist = _dist()
+        if _staged(self.buf, self.group):
+            if self._host is None:
+                self._host = (torch.empty_like(self.buf, device="cpu").pin_memory(),
+                              torch.empty_like(self.mine, device="cpu").pin_memory())
+            hb, hm = self._host
+            hm.copy_(self.mine)
+            dist.all_gather_into_tensor(hb, hm, group=self.group)
+            self.buf.copy_(hb, non_blocking=False)
+        else:
+            # in place: the input is this rank's block of the output buffer
+            dist.all_gather_into_tensor(self.buf, self.mine, group=self.group)
+
+
+def allreduce_(t: torch.Tensor, world: int, group=None):
+    """In-place sum over ranks (a few bytes: flags, the dangling mass)."""
+    if world == 1:
+        return
+    dist = _dist()
+    if _staged(t, group):
+        h = t.cpu()
+        dist.all_reduce(h, group=group)
+        t.copy_(h)
+    else:
+        dist.all_reduce(t, group=group)
+
+
+class HaloRows:
+    """Halo rows of a W x H row-slab decomposition (GEN).
+
+    Rank r owns rows [r0, r1). Before a generation it needs rows r0-1 and r1
+    (torus: modulo H) of the previous state, owned by the neighbour slabs.
+    ``exchange(state)`` sends its first / last owned row to the previous /
+    next rank and receives theirs into the halo rows of `state` (a full-size
+    H*W uint8 buffer indexed by global cell)."""
+
+    def __init__(self, W: int, H: int, rank: int, world: int, torus: bool = False, group=None):
+        self.W, self.H, self.rank, self.world, self.torus, self.group = W, H, rank, world, torus, group
+        self.r0, self.r1, self.per = block_range(H, rank, world)
+        self._host = None
+
+    def _peers(self):
+        prev = self.rank - 1 if self.rank > 0 else (self.world - 1 if self.torus else None)
+        nxt = self.rank + 1 if self.rank < self.world - 1 else (0 if self.torus else None)
+        return prev, nxt
+
+    def exchange(self, state: torch.Tensor):
+        if self.world == 1 or self.r1 <= self.r0:
+            return
+        dist = _dist()
+        W, H = self.W, self.H
+        s2 = state.view(H, W)
+        prev, nxt = self._peers()
+        staged = _staged(state, self.group)
+        if staged:
+            if self._host is None:
+                self._host = [torch.empty(W, dtype=state.dtype).pin_memory() for _ in range(4)]
+            send_first, send_last, recv_above, recv_below = self._host
+            send_first.copy_(s2[self.r0])
+            send_last.copy_(s2[self.r1 - 1])
+        else:
+            send_first, send_last = s2[self.r0], s2[self.r1 - 1]
+            recv_above = s2[(self.r0 - 1) % H]
+            recv_below = s2[self.r1 % H]
+        # downward messages (last row -> next slab's halo above) first, then
+        # upward ones: messages between one pair of ranks match in posting
+        # order, which keeps world = 2 with torus (both neighbours are the same
+        # rank) correct
+        ops = []
+        g = self.group
+        if nxt is not None:
+            ops.append(dist.P2POp(dist.isend, send_last, _peer_global(nxt, g), g))
+        if prev is not None:
+            ops.append(dist.P2POp(dist.irecv, recv_above, _peer_global(prev, g), g))
+            ops.append(dist.P2POp(dist.isend, send_first, _peer_global(prev, g), g))
+        if nxt is not None:
+            ops.append(dist.P2POp(dist.irecv, recv_below, _peer_global(nxt, g), g))
+        if ops:
+            for r in dist.batch_isend_irecv(ops):
+                r.wait()
+        if staged:
+            if prev is not None:
+                s2[(self.r0 - 1) % H].copy_(recv_above)
+            if nxt is not None:
+                s2[self.r1 % H].copy_(recv_below)
+
+
+def _peer_global(r: int, group):
+    if group is None:
+        return r
+    return _dist().get_global_rank(group, r)

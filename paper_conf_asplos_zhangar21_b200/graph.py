@@ -20,7 +20,7 @@ import torch
 
 import synth
 
-from . import vf
+from . import exchange, vf
 
 
 def _sync_scalar(t):
@@ -28,30 +28,33 @@ def _sync_scalar(t):
 
 
 def block_range(V: int, rank: int, world: int):
-    """Owned vertex block [lo, hi) of `rank` and the per-rank block size."""
-    per = (V + world - 1) // world
-    return min(V, rank * per), min(V, (rank + 1) * per), per
+    """Owned vertex block [lo, hi) of `rank` and the per-rank block size (a
+    multiple of 32 for world > 1, so frontier-bitmap slices are whole u32 words)."""
+    return exchange.block_range(V, rank, world, align=32 if world > 1 else 1)
 
 
 def allgather_block(t, V: int, per: int, rank: int, world: int, group=None):
-    """In-place all-gather of each rank's owned block of a per-vertex array (§8e):
-    after the call every rank holds every rank's block."""
+    """All-gather of each rank's owned block of a per-vertex array held in a
+    plain (unpadded) tensor: kept for callers outside the app classes, which
+    use persistent padded ``exchange.BlockArray`` buffers instead."""
     if world == 1:
         return
     import torch.distributed as dist
-    rest = tuple(t.shape[1:])  # per-vertex rows (e.g. float4 positions)
+    rest = tuple(t.shape[1:])
     padded = torch.zeros((per * world,) + rest, dtype=t.dtype, device=t.device)
     padded[:V] = t
-    out = [torch.empty((per,) + rest, dtype=t.dtype, device=t.device) for _ in range(world)]
-    dist.all_gather(out, padded[rank * per:(rank + 1) * per].clone(), group=group)
-    t.copy_(torch.cat(out)[:V])
+    mine = padded[rank * per:(rank + 1) * per].clone()
+    if exchange._staged(padded, group):
+        h = padded.cpu()
+        dist.all_gather_into_tensor(h, mine.cpu(), group=group)
+        padded.copy_(h)
+    else:
+        dist.all_gather_into_tensor(padded, mine, group=group)
+    t.copy_(padded[:V])
 
 
 def allreduce_sum(t, world: int, group=None):
-    if world == 1:
-        return
-    import torch.distributed as dist
-    dist.all_reduce(t, group=group)
+    exchange.allreduce_(t, world, group)
 
 
 def work_entries(deg: np.ndarray, lo: int, hi: int, C: int):
@@ -88,10 +91,7 @@ class Graph:
         ctor = np.stack([own.astype(np.uint32), deg[own].astype(np.uint32)], axis=1).copy()
         ctor_t = torch.from_numpy(ctor.view(np.int32)).to(dev)
         tt = torch.from_numpy(types[own].astype(np.int32)).to(dev)
-        if variant == "cuda":
-            objs = ctx.alloc_cuda(vf.APP_GRAPH, tt, ctor_t)
-        else:
-            objs = ctx.alloc_typed_batch(vf.APP_GRAPH, tt, ctor_t, tag=(variant == "typeptr"))
+        objs = ctx.alloc_for(variant, vf.APP_GRAPH, tt, ctor_t)
         # vobj is indexed by global vertex id; only the owned block is filled on this rank
         self.vobj = torch.zeros(V, dtype=torch.int64, device=dev)
         self.vobj[self.lo:self.hi] = objs
@@ -102,14 +102,24 @@ class Graph:
         self.entries = self.vobj[torch.from_numpy(evid).to(dev)].contiguous()
         self.entry_chunk = torch.from_numpy(ech.view(np.int32)).to(dev)
         e_all = int(np.maximum(1, (deg + self.C - 1) // self.C).sum())
-        self.depth = torch.empty(V, dtype=torch.int32, device=dev)
+        # per-vertex state in persistent buffers padded to per * world rows; the
+        # owned block of each is all-gathered in place (exchange.BlockArray)
+        blk = dict(n=V, per=self.per, rank=rank, world=world, device=dev, group=group)
+        self._depth = exchange.BlockArray(dtype=torch.int32, **blk)
+        self.depth = self._depth.view
+        nw = (V + 31) // 32
+        wblk = dict(n=nw, per=self.per // 32 if world > 1 else nw, rank=rank, world=world, device=dev, group=group)
+        self._bits = [exchange.BlockArray(dtype=torch.int32, **wblk) for _ in range(2)]
         self.q = [torch.empty(max(e_all, 1), dtype=torch.int64, device=dev) for _ in range(2)]
         self.qc = [torch.empty(max(e_all, 1), dtype=torch.int32, device=dev) for _ in range(2)]
         self.count = torch.zeros(1, dtype=torch.int32, device=dev)
-        self.lab = [torch.empty(V, dtype=torch.int32, device=dev) for _ in range(2)]
+        self._lab = [exchange.BlockArray(dtype=torch.int32, **blk) for _ in range(2)]
+        self.lab = [b.view for b in self._lab]
         self.changed = torch.zeros(1, dtype=torch.int32, device=dev)
-        self.rk = [torch.empty(V, dtype=torch.float32, device=dev) for _ in range(2)]
-        self.contrib = torch.empty(V, dtype=torch.float64, device=dev)
+        self._rk = [exchange.BlockArray(dtype=torch.float32, **blk) for _ in range(2)]
+        self.rk = [b.view for b in self._rk]
+        self._contrib = exchange.BlockArray(dtype=torch.float64, **blk)
+        self.contrib = self._contrib.view
         self.dangling = torch.zeros(1, dtype=torch.float64, device=dev)
         self.partial = torch.zeros(max(self.E, 1), dtype=torch.float64, device=dev)
         self.counter = torch.zeros(V, dtype=torch.int32, device=dev)
@@ -117,11 +127,8 @@ class Graph:
         torch.cuda.synchronize(dev)
 
     # ---------------------------------------------------------------- helpers
-    def _allgather_block(self, t):
-        allgather_block(t, self.V, self.per, self.rank, self.world, self.group)
-
     def _allreduce_sum(self, t):
-        allreduce_sum(t, self.world, self.group)
+        exchange.allreduce_(t, self.world, self.group)
 
     def _dispatch(self, method, objs_ptr, n, args, stream=None):
         st = self.ctx.dispatch_raw(self.v, vf.APP_GRAPH, method, objs_ptr, n, args, vf._stream(stream))
@@ -133,7 +140,9 @@ class Graph:
         """Level-synchronous BFS from src; returns (depth tensor, levels, calls).
         topdown: one virtual bfs_expand() per frontier work entry (single GPU);
         hybrid: top-down, then bottom-up once the frontier exceeds V / alpha entries (single GPU);
-        bottomup: one virtual bfs_probe() per owned work entry per level (multi-GPU)."""
+        bottomup: one virtual bfs_probe() per work entry per level, depth array as frontier (single GPU);
+        bits (and every mode at world > 1): one virtual bfs_probe_bits() per owned work entry per
+        level over a frontier bitmap whose owned slices are all-gathered (multi-GPU)."""
         L = vf.lib()
         st = L.vf_graph_bfs_init(self.V, self.depth.data_ptr(), src, self.vobj.data_ptr(), self.offs.data_ptr(),
                                  self.C, self.q[0].data_ptr(), self.qc[0].data_ptr(), self.count.data_ptr(),
@@ -179,7 +188,7 @@ class Graph:
                 self.q[0], self.q[1] = self.q[1], self.q[0]
                 self.qc[0], self.qc[1] = self.qc[1], self.qc[0]
                 level += 1
-        else:
+        elif mode == "bottomup" and self.world == 1:
             while True:
                 self.count.zero_()
                 a = vf.graph_bfs_args(self.offs.data_ptr(), self.col.data_ptr(), self.depth.data_ptr(),
@@ -187,13 +196,43 @@ class Graph:
                                       level, self.C)
                 self._dispatch(vf.GRAPH_BFS_PROBE, self.entries.data_ptr(), self.E, a)
                 calls += self.E
-                self._allreduce_sum(self.count)
-                self._allgather_block(self.depth)
                 level += 1
                 if _sync_scalar(self.count) == 0:
                     break
+        else:
+            level, calls = self._bfs_bits(src)
         self.calls = calls
         return self.depth, level, calls
+
+    def _bfs_bits(self, src: int):
+        """Bottom-up BFS over frontier bitmaps (multi-GPU): per level
+        one virtual bfs_probe_bits() per owned work entry, then ONE all-gather of
+        the owned bitmap slices (V/8 bytes in total) and an all-reduce of the
+        "joined" flag. Depths stay on their owner until the end."""
+        cur, nxt = self._bits
+        cur.view.zero_()
+        word, bit = divmod(src, 32)
+        cur.view[word] = int(np.array(1 << bit, dtype=np.uint32).view(np.int32))
+        if self.lo <= src < self.hi:
+            self.depth[src] = 0
+        calls, level = 0, 0
+        while True:
+            nxt.mine.zero_()
+            self.count.zero_()
+            a = vf.graph_bfs_bits_args(self.offs.data_ptr(), self.col.data_ptr(), self.depth.data_ptr(),
+                                       cur.data_ptr(), nxt.data_ptr(), self.entry_chunk.data_ptr(),
+                                       self.count.data_ptr(), level, self.C)
+            self._dispatch(vf.GRAPH_BFS_PROBE_BITS, self.entries.data_ptr(), self.E, a)
+            calls += self.E
+            self._allreduce_sum(self.count)
+            nxt.gather()
+            cur, nxt = nxt, cur
+            level += 1
+            if _sync_scalar(self.count) == 0:
+                break
+        self._bits = [cur, nxt]
+        self._depth.gather()
+        return level, calls
 
     # ---------------------------------------------------------------- CC
     def cc(self, max_iters: int = 10 ** 6):
@@ -209,9 +248,10 @@ class Graph:
             self._dispatch(vf.GRAPH_CC_UPDATE, self.entries.data_ptr(), self.E, a)
             calls += self.E
             it += 1
-            self._allgather_block(self.lab[1])
+            self._lab[1].gather()
             self._allreduce_sum(self.changed)
-            self.lab[0], self.lab[1] = self.lab[1], self.lab[0]
+            self._lab.reverse()
+            self.lab = [b.view for b in self._lab]
             if _sync_scalar(self.changed) == 0:
                 break
         self.calls = calls
@@ -228,11 +268,11 @@ class Graph:
                              self.contrib.data_ptr(), self.dangling.data_ptr(), (1.0 - d) / self.V, d, float(self.V),
                              self.entry_chunk.data_ptr(), self.partial.data_ptr(), self.counter.data_ptr(), self.C)
         self._dispatch(vf.GRAPH_PR_CONTRIB, self.entries.data_ptr(), self.E, a, stream)
-        self._allgather_block(self.contrib)
+        self._contrib.gather()
         self._allreduce_sum(self.dangling)
         self._dispatch(vf.GRAPH_PR_UPDATE, self.entries.data_ptr(), self.E, a, stream)
-        self._allgather_block(self.rk[1])
-        self.rk[0], self.rk[1] = self.rk[1], self.rk[0]
+        self._rk.reverse()
+        self.rk = [b.view for b in self._rk]
         return 2 * self.E
 
     def pagerank(self, iters: int = 20, d: float = 0.85):
@@ -240,5 +280,6 @@ class Graph:
         calls = 0
         for _ in range(iters):
             calls += self.pr_iteration(d)
+        self._rk[0].gather()  # ranks stay on their owner during the iterations
         self.calls = calls
         return self.rk[0], calls

@@ -16,8 +16,8 @@ import ctypes
 import numpy as np
 import torch
 
-from . import vf
-from .graph import allgather_block, block_range
+from . import exchange as xc, vf
+from .exchange import block_range
 
 
 class Nbody:
@@ -38,12 +38,14 @@ class Nbody:
         ctor[:, 1:] = np.ascontiguousarray(sys_["vel"][own], dtype=np.float32).view(np.uint32)
         tt = torch.from_numpy(sys_["types"][own].astype(np.int32)).to(dev)
         ct = torch.from_numpy(ctor.view(np.int32)).to(dev)
-        if variant == "cuda":
-            self.objs = ctx.alloc_cuda(vf.APP_NBODY, tt, ct)
-        else:
-            self.objs = ctx.alloc_typed_batch(vf.APP_NBODY, tt, ct, tag=(variant == "typeptr"))
+        self.objs = ctx.alloc_for(variant, vf.APP_NBODY, tt, ct)
         pos = torch.from_numpy(np.ascontiguousarray(sys_["pos"], dtype=np.float32)).to(dev)
-        self.p = [pos.clone(), torch.zeros_like(pos)]
+        # double-buffered positions in persistent buffers padded to per * world
+        # rows; the owned block of the new buffer is all-gathered in place
+        self._p = [xc.BlockArray(N, self.per, rank, world, torch.float32, dev, rest=(4,), group=group, fill=0.0)
+                   for _ in range(2)]
+        self._p[0].view.copy_(pos)
+        self.p = [b.view for b in self._p]
         self.dt = float(sys_["dt"])
         self.eps2 = [float(x) for x in sys_["eps2"]]
         self.damp = float(sys_["damp"])
@@ -64,8 +66,9 @@ class Nbody:
         if st:
             self.ctx._check(st, "nbody update")
         if self.world > 1 and self.exchange:
-            allgather_block(self.p[1], self.N, self.per, self.rank, self.world, self.group)
-        self.p[0], self.p[1] = self.p[1], self.p[0]
+            self._p[1].gather()
+        self._p.reverse()
+        self.p = [b.view for b in self._p]
 
     def positions(self):
         return self.p[0].cpu().numpy()

@@ -3,8 +3,9 @@
 Allocates the scene's shape objects through libvf (typed arenas / device heap)
 and renders with vf_ray_render. Multi-GPU: 8-row pixel strips are dealt
 round-robin to ranks (§8e); each rank renders its strips (independent, no
-data-path collective) and the image is all-gathered once at the end, outside
-the timed calls/s.
+data-path collective) and the image is assembled once at the end
+(Ray.gather_image: one all-reduce each of rgb and hit ids), outside the timed
+calls/s.
 """
 from __future__ import annotations
 
@@ -29,10 +30,7 @@ class Ray:
         self.S = len(types)
         tt = torch.from_numpy(np.asarray(types, np.int32)).to(dev)
         pp = torch.from_numpy(np.ascontiguousarray(params, np.float32)).to(dev)
-        if variant == "cuda":
-            self.objs = ctx.alloc_cuda(vf.APP_RAY, tt, pp)
-        else:
-            self.objs = ctx.alloc_typed_batch(vf.APP_RAY, tt, pp, tag=(variant == "typeptr"))
+        self.objs = ctx.alloc_for(variant, vf.APP_RAY, tt, pp)
         self.albedo = (ctypes.c_float * 12)(*synth.RAY_ALBEDO.reshape(-1).tolist())
         torch.cuda.synchronize(dev)
 
@@ -60,8 +58,31 @@ class Ray:
             k += 1
         return out
 
+    @staticmethod
+    def gather_image(rgb, hid, world: int, group=None):
+        """Assemble the frame on every rank after render_frame (once
+        per frame, outside the timed calls/s). Rows a rank does not own hold
+        rgb 0 and hit id -1, so one SUM all-reduce of rgb (x + 0 = x exactly)
+        and one MAX all-reduce of the hit ids (-1 < any id) give every rank the
+        whole image."""
+        if world == 1:
+            return rgb, hid
+        import torch.distributed as dist
+        from . import exchange
+        if exchange._staged(rgb, group):
+            hr, hh = rgb.cpu(), hid.cpu()
+            dist.all_reduce(hr, group=group)
+            dist.all_reduce(hh, op=dist.ReduceOp.MAX, group=group)
+            rgb.copy_(hr)
+            hid.copy_(hh)
+        else:
+            dist.all_reduce(rgb, group=group)
+            dist.all_reduce(hid, op=dist.ReduceOp.MAX, group=group)
+        return rgb, hid
+
     def render_frame(self, W: int, H: int, cam, rank: int = 0, world: int = 1, rgb=None, hid=None, stream=None):
-        """Render this rank's strips into full-frame buffers (rows it does not own untouched)."""
+        """Render this rank's strips into full-frame buffers (rows it does not own
+        keep rgb 0 / hit id -1; gather_image assembles the frame)."""
         if rgb is None:
             rgb = torch.zeros((H, W, 3), dtype=torch.float32, device=self.dev)
         if hid is None:

@@ -15,8 +15,8 @@ from __future__ import annotations
 import numpy as np
 import torch
 
-from . import vf
-from .graph import allgather_block, block_range
+from . import exchange as xc, vf
+from .exchange import block_range
 
 
 class Stut:
@@ -53,14 +53,11 @@ class Stut:
         st = torch.full((len(sids),), 3, dtype=torch.int32, device=dev)
         nc = torch.from_numpy(nctor.view(np.int32)).to(dev)
         sc = torch.from_numpy(sctor.view(np.int32)).to(dev)
-        if variant == "cuda":
-            self.nodes = ctx.alloc_cuda(vf.APP_STUT, nt, nc)
-            self.springs = ctx.alloc_cuda(vf.APP_STUT, st, sc)
-        else:
-            tag = variant == "typeptr"
-            self.nodes = ctx.alloc_typed_batch(vf.APP_STUT, nt, nc, tag=tag)
-            self.springs = ctx.alloc_typed_batch(vf.APP_STUT, st, sc, tag=tag)
-        self.pos = torch.from_numpy(np.ascontiguousarray(w["pos"], np.float32)).to(dev)
+        self.nodes = ctx.alloc_for(variant, vf.APP_STUT, nt, nc)
+        self.springs = ctx.alloc_for(variant, vf.APP_STUT, st, sc)
+        self._pos = xc.BlockArray(n, self.per, rank, world, torch.float32, dev, rest=(2,), group=group, fill=0.0)
+        self._pos.view.copy_(torch.from_numpy(np.ascontiguousarray(w["pos"], np.float32)))
+        self.pos = self._pos.view
         self.F = torch.zeros((max(S, 1), 2), dtype=torch.float32, device=dev)
         self.inc_offs = torch.from_numpy(np.ascontiguousarray(w["inc_offs"], np.uint32).view(np.int32)).to(dev)
         self.inc = torch.from_numpy(np.ascontiguousarray(w["inc"], np.uint32).view(np.int32)).to(dev)
@@ -85,7 +82,7 @@ class Stut:
         if st:
             self.ctx._check(st, "stut move")
         if self.world > 1 and self.exchange:
-            allgather_block(self.pos, self.n, self.per, self.rank, self.world, self.group)
+            self._pos.gather()
 
     def positions(self):
         return self.pos.cpu().numpy()

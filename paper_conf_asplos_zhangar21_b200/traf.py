@@ -43,12 +43,8 @@ class Traf:
         vargs[:, 1] = world["veh_ring"][vsel] - r0
         vargs[:, 2] = world["veh_pos"][vsel]
         veh_args = torch.from_numpy(vargs.view(np.int32)).to(dev)
-        if variant == "cuda":
-            self.cells = ctx.alloc_cuda(vf.APP_TRAF, cell_types, cell_args)
-            self.vehs = ctx.alloc_cuda(vf.APP_TRAF, veh_types, veh_args)
-        else:
-            self.cells = ctx.alloc_typed_batch(vf.APP_TRAF, cell_types, cell_args, tag=tag)
-            self.vehs = ctx.alloc_typed_batch(vf.APP_TRAF, veh_types, veh_args, tag=tag)
+        self.cells = ctx.alloc_for(variant, vf.APP_TRAF, cell_types, cell_args)
+        self.vehs = ctx.alloc_for(variant, vf.APP_TRAF, veh_types, veh_args)
         self.occ = [torch.zeros(N, dtype=torch.uint8, device=dev) for _ in range(2)]
         self.blocked = torch.zeros(N, dtype=torch.uint8, device=dev)
         self.seed = world["seed"]

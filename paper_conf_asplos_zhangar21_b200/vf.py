@@ -18,13 +18,15 @@ SO = os.path.join(PKG, "libvf.so")
 # enums mirrored from include/vf.h
 VF_OK = 0
 CUDA, SHAREDOA, COAL, TYPEPTR, CONCORD = 0, 1, 2, 3, 4
-VARIANTS = {"cuda": CUDA, "sharedoa": SHAREDOA, "coal": COAL, "typeptr": TYPEPTR, "concord": CONCORD}
+VARIANTS = {"cuda": CUDA, "sharedoa": SHAREDOA, "coal": COAL, "typeptr": TYPEPTR, "concord": CONCORD,
+            "cuda_packed": CUDA}  # cuda_packed: CUDA dispatch over an index-ordered slab (vf_alloc_packed)
 ORDERS = {"random": 0, "sorted": 1, "kperwarp": 2}
 APP_MICRO, APP_GOL, APP_GEN, APP_GRAPH = 0, 1, 2, 3
 MICRO_APPLY, MICRO_GET = 0, 1
 GOL_NEXT, GOL_GET = 0, 1
 GEN_NEXT, GEN_GET = 0, 1
 GRAPH_BFS_EXPAND, GRAPH_BFS_PROBE, GRAPH_CC_UPDATE, GRAPH_PR_CONTRIB, GRAPH_PR_UPDATE = 0, 1, 2, 3, 4
+GRAPH_BFS_PROBE_BITS = 5
 NOT_FOUND = 0xFFFFFFFF
 VA_BITS = 57
 MAX_RANGES = 4096
@@ -35,11 +37,11 @@ STATUS = {0: "VF_OK", 1: "VF_ERR_INVALID", 2: "VF_ERR_OOM", 3: "VF_ERR_CUDA", 4:
 # exported symbols (checked by tests/test_abi.py against include/vf.h)
 SYMBOLS = [
     "vf_config_default", "vf_create", "vf_destroy", "vf_status_str", "vf_last_error", "vf_app_info",
-    "vf_alloc_typed", "vf_alloc_typed_batch", "vf_alloc_cuda", "vf_reset", "vf_range_table",
+    "vf_alloc_typed", "vf_alloc_typed_batch", "vf_alloc_cuda", "vf_alloc_packed", "vf_reset", "vf_range_table",
     "vf_regions", "vf_type_vptrs", "vf_resolve", "vf_verify_types", "vf_dispatch_cuda",
     "vf_dispatch_sharedoa", "vf_dispatch_coal", "vf_dispatch_typeptr", "vf_dispatch",
     "vf_gol_neighbors", "vf_gol_swap", "vf_gen_swap", "vf_checksum_i32", "vf_launch_count", "vf_set_tuning",
-    "vf_graph_bfs_init", "vf_iota_u32", "vf_fill_f32", "vf_ray_render", "vf_gol_step", "vf_gen_step", "vf_gol_run", "vf_dispatch_host",
+    "vf_graph_bfs_init", "vf_iota_u32", "vf_fill_f32", "vf_ray_render", "vf_gol_step", "vf_gen_step", "vf_gen_step_rows", "vf_gol_run", "vf_dispatch_host",
     "vf_dispatch_concord", "vf_micro_branch", "vf_collide_tmp_words", "vf_collide_grid",
 ]
 APP_RAY = 4
@@ -212,6 +214,12 @@ class graph_bfs_args(ctypes.Structure):
                 ("C", ctypes.c_uint32)]
 
 
+class graph_bfs_bits_args(ctypes.Structure):
+    _fields_ = [("offs_dev", ctypes.c_void_p), ("col_dev", ctypes.c_void_p), ("depth_dev", ctypes.c_void_p),
+                ("frontier_dev", ctypes.c_void_p), ("next_dev", ctypes.c_void_p), ("chunk_dev", ctypes.c_void_p),
+                ("next_count_dev", ctypes.c_void_p), ("level", ctypes.c_int32), ("C", ctypes.c_uint32)]
+
+
 class graph_cc_args(ctypes.Structure):
     _fields_ = [("offs_dev", ctypes.c_void_p), ("col_dev", ctypes.c_void_p), ("label_in_dev", ctypes.c_void_p),
                 ("label_out_dev", ctypes.c_void_p), ("changed_dev", ctypes.c_void_p), ("chunk_dev", ctypes.c_void_p),
@@ -248,6 +256,7 @@ def lib(required: bool = True):
         "vf_alloc_typed": (I, [P, U32, U32, U64, P, U32, P, I, P]),
         "vf_alloc_typed_batch": (I, [P, U32, P, U64, P, U32, P, I, P]),
         "vf_alloc_cuda": (I, [P, U32, P, U64, P, U32, P, I, P]),
+        "vf_alloc_packed": (I, [P, U32, P, U64, P, U32, P, P]),
         "vf_reset": (I, [P]),
         "vf_range_table": (I, [P, U32, ctypes.POINTER(ctypes.POINTER(vf_range)), ctypes.POINTER(U32)]),
         "vf_regions": (I, [P, ctypes.POINTER(ctypes.POINTER(vf_region)), ctypes.POINTER(U32)]),
@@ -277,6 +286,7 @@ def lib(required: bool = True):
         "vf_collide_tmp_words": (U64, [U32, U32]),
         "vf_collide_grid": (I, [ctypes.POINTER(collide_grid_args), P]),
         "vf_gen_step": (I, [P, I, U32, U32, I, P, P, P, P, P, P, P, U32, U32, U32, P]),
+        "vf_gen_step_rows": (I, [P, I, U32, U32, I, U32, U32, P, P, P, P, P, P, P, U32, U32, U32, P]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)
@@ -398,6 +408,26 @@ class Ctx:
                                          int(tag), _stream(stream)), "alloc_cuda")
         return out
 
+    def alloc_packed(self, app, types, ctor_args=None, stream=None):
+        """cuda_packed: placement into one index-ordered slab (dispatch with CUDA)."""
+        import torch
+        n = types.numel()
+        out = torch.empty(n, dtype=torch.int64, device=types.device)
+        ab = 0 if ctor_args is None else ctor_args.element_size() * (ctor_args.numel() // max(n, 1))
+        self._check(self.L.vf_alloc_packed(self.h, app, _ptr(types), n, _ptr(ctor_args), ab, _ptr(out),
+                                           _stream(stream)), "alloc_packed")
+        return out
+
+    def alloc_for(self, variant: str, app, types, ctor_args=None, stream=None):
+        """The allocation each dispatch variant runs on: device-heap `new` (cuda),
+        one index-ordered slab (cuda_packed), or the typed arenas (sharedoa /
+        coal / concord untagged, typeptr tagged)."""
+        if variant == "cuda":
+            return self.alloc_cuda(app, types, ctor_args, stream=stream)
+        if variant == "cuda_packed":
+            return self.alloc_packed(app, types, ctor_args, stream=stream)
+        return self.alloc_typed_batch(app, types, ctor_args, tag=(variant == "typeptr"), stream=stream)
+
     def reset(self):
         self._check(self.L.vf_reset(self.h), "reset")
 
@@ -496,6 +526,15 @@ def gen_step(ctx: Ctx, variant: int, W, H, torus, prev, nxt, nbr, grid, dead, al
                            _ptr(dead), _ptr(alive), _ptr(dying), born, survive, C, _stream(stream))
     if st:
         ctx._check(st, "gen_step")
+
+
+def gen_step_rows(ctx: Ctx, variant: int, W, H, torus, row0, nrows, prev, nxt, nbr, grid, dead, alive, dying,
+                  born, survive, C, stream=None):
+    st = lib().vf_gen_step_rows(ctx.h, variant, W, H, int(torus), row0, nrows, _ptr(prev), _ptr(nxt), _ptr(nbr),
+                                _ptr(grid), _ptr(dead), _ptr(alive), _ptr(dying), born, survive, C,
+                                _stream(stream))
+    if st:
+        ctx._check(st, "gen_step_rows")
 
 
 def micro_branch(vals, T: int, order: str, seed: int, k: int = 1, stream=None):

@@ -162,3 +162,62 @@ def test_ray_strips_tile_the_frame():
         for rank in range(world):
             rows += [r for r0, n in Ray.strips(Ray, H, rank, world) for r in range(r0, r0 + n)]
         assert sorted(rows) == list(range(H))
+
+
+def _exchange_worker(rank, world, port, outdir):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    from paper_conf_asplos_zhangar21_b200 import exchange
+    out = {}
+    # BlockArray: padded persistent buffer, each rank writes its block, one gather
+    n = 101
+    lo, hi, per = exchange.block_range(n, rank, world, align=8)
+    ba = exchange.BlockArray(n, per, rank, world, torch.float64, "cpu", rest=(3,), fill=-1.0)
+    ptr = ba.data_ptr()
+    for it in range(3):  # persistent: repeated gathers reuse the same storage
+        ba.view[lo:hi] = torch.arange(lo, hi, dtype=torch.float64)[:, None] * (it + 1) + torch.arange(3)
+        ba.gather()
+    assert ba.data_ptr() == ptr
+    out["ba"] = ba.view.numpy().copy()
+    # halo rows of a W x H row-slab decomposition, dead border and torus
+    W, H = 5, 11
+    for torus in (False, True):
+        h = exchange.HaloRows(W, H, rank, world, torus)
+        st = torch.full((H * W,), 255, dtype=torch.uint8)
+        rows = torch.arange(H, dtype=torch.uint8)[:, None].expand(H, W).reshape(-1)
+        st[h.r0 * W:h.r1 * W] = rows[h.r0 * W:h.r1 * W]
+        h.exchange(st)
+        out[f"halo{int(torus)}"] = st.numpy().copy()
+        out[f"r{int(torus)}"] = np.array([h.r0, h.r1])
+    c = torch.tensor([rank + 1.5], dtype=torch.float64)
+    exchange.allreduce_(c, world)
+    out["sum"] = c.numpy()
+    np.savez(os.path.join(outdir, f"x{rank}.npz"), **out)
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_exchange_blockarray_halo_gloo(world):
+    """exchange.py (the GPU apps' data plane) over real gloo groups: one
+    in-place all-gather of padded blocks into a persistent buffer, the GEN
+    halo rows (dead border and torus, incl. world 2 where both neighbours are
+    the same rank), and the scalar all-reduce."""
+    with tempfile.TemporaryDirectory() as td:
+        mp.spawn(_exchange_worker, args=(world, _free_port(), td), nprocs=world, join=True)
+        res = [dict(np.load(os.path.join(td, f"x{r}.npz"))) for r in range(world)]
+    n = 101
+    expect = np.arange(n, dtype=np.float64)[:, None] * 3 + np.arange(3)
+    W, H = 5, 11
+    for r in res:
+        assert np.array_equal(r["ba"], expect)
+        assert r["sum"][0] == sum(k + 1.5 for k in range(world))
+        for torus in (0, 1):
+            r0, r1 = r[f"r{torus}"]
+            st = r[f"halo{torus}"].reshape(H, W)
+            assert (st[r0:r1] == np.arange(r0, r1)[:, None]).all()
+            for row in (r0 - 1, r1):
+                if 0 <= row < H or torus:
+                    assert (st[row % H] == row % H).all(), (torus, row)
+            untouched = [q for q in range(H) if not (r0 - 1 <= q <= r1) and not (torus and q in ((r0 - 1) % H, r1 % H))]
+            assert all((st[q] == 255).all() for q in untouched)
