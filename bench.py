@@ -46,8 +46,12 @@ def parse():
     ap.add_argument("--order", default="random", choices=["random", "sorted", "kperwarp"])
     ap.add_argument("--n", type=int, default=1 << 26)
     ap.add_argument("--seed", type=int, default=42)
-    ap.add_argument("--cuda-n", type=int, default=1 << 22,
-                    help="objects for the device-heap CUDA baseline (device `new` of 2^26 objects takes minutes)")
+    ap.add_argument("--cuda-n", type=int, default=1 << 24,
+                    help="objects for the same-config comparison with the device-heap CUDA baseline (device "
+                         "`new` of 2^24 objects takes ~36 s on B200, of 2^26 ~10 min)")
+    ap.add_argument("--apps", default=",".join(("gol", "ray", "nbody", "gen", "traf", "stut", "collide", "graph")),
+                    help="per-app block (BASELINE configs 1, 3, 4, 5); '' to skip")
+    ap.add_argument("--app-variants", default="cuda,cuda_packed,sharedoa,coal,typeptr")
     ap.add_argument("--no-variants", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
@@ -200,7 +204,7 @@ def run_ours(args, rank, world, local):
 
     torch.cuda.set_device(local)
     dev = torch.device(f"cuda:{local}")
-    ctx = vf.Ctx(local, cuda_heap_bytes=8 << 30)
+    ctx = vf.Ctx(local, cuda_heap_bytes=16 << 30)
     s = torch.cuda.Stream(device=dev)
     n = args.n
     types = synth.micro_types(n, args.T, args.order, seed=args.seed + rank)
@@ -317,7 +321,7 @@ def run_ours(args, rank, world, local):
 
     # ---- the other variants (same config; device-heap CUDA baseline at cuda_n) ----
     if not args.no_variants:
-        for variant in ("sharedoa", "coal", "typeptr"):
+        for variant in ("cuda_packed", "sharedoa", "coal", "typeptr"):
             if variant == args.variant:
                 results[variant] = {"calls_per_s": value, "n": n}
                 continue
@@ -329,7 +333,7 @@ def run_ours(args, rank, world, local):
         # device-heap `new` baseline (paper's CUDA) at a size it allocates in seconds
         cn = min(args.cuda_n, n)
         small = {}
-        for variant in ("cuda", "sharedoa", "coal", "typeptr"):
+        for variant in ("cuda", "cuda_packed", "sharedoa", "coal", "typeptr"):
             mv = apps.Micro(ctx, cn, args.T, variant=variant, types_np=types[:cn], init_np=init[:cn])
             vms = timed_flush(mv, 30, args.warmup)
             small[variant] = world * cn * 30 / (vms / 1e3)
@@ -341,7 +345,10 @@ def run_ours(args, rank, world, local):
         base = results.get("sharedoa", {}).get("calls_per_s")
         if base:
             results["speedup_vs_sharedoa_at_n"] = {k: results[k]["calls_per_s"] / base
-                                                   for k in ("sharedoa", "coal", "typeptr")}
+                                                   for k in ("cuda_packed", "sharedoa", "coal", "typeptr")}
+        if results.get("cuda_packed"):
+            results["speedup_vs_cuda_packed_at_n"] = {k: results[k]["calls_per_s"] / results["cuda_packed"]["calls_per_s"]
+                                                      for k in ("cuda_packed", "sharedoa", "coal", "typeptr")}
 
     # ---- CPU baseline: the oracle on this host, bounded sample (rank 0, N=1 only) ----
     cpu = None
@@ -354,6 +361,22 @@ def run_ours(args, rank, world, local):
         cpu = {"value": n_s * reps_c / sec, "unit": "calls/s", "cores": threads, "kind": "oracle",
                "sample": f"{n_s} objects x {reps_c} passes ({args.order}, T={args.T}), OpenMP {threads} "
                          f"threads, {cpu_model()}"}
+
+    # ---- per-app block: BASELINE configs 1, 3, 4, 5 (tools/apps_bench.py) ----
+    apps_block = None
+    names = [a for a in args.apps.split(",") if a]
+    if names:
+        sys.path.insert(0, os.path.join(ROOT, "tools"))
+        import apps_bench
+        env = apps_bench.Env(ctx, rank, world, None, local)
+
+        def log(name, row):
+            if rank == 0:
+                print(f"# app {name}: {row.get('wall_s', 0):.1f} s", file=sys.stderr, flush=True)
+
+        apps_block = apps_bench.run_apps(env, names, tuple(args.app_variants.split(",")),
+                                         cpu=(rank == 0 and world == 1 and not args.no_cpu), clocks_cls=Clocks,
+                                         log=log)
 
     pk = peaks()
     hbm = pk.get("hbm_gbs")
@@ -380,7 +403,7 @@ def run_ours(args, rank, world, local):
                "vs_baseline": None, "dtype": "int32", "data": "synthetic",
                "config": workload_config(args, world),
                "gpu_launches": launches, "parity_sample_ok": ok, "roofline": roof, "clocks": clk,
-               "e2e": e2e, "cpu_baseline": cpu, "variants": results}
+               "e2e": e2e, "cpu_baseline": cpu, "variants": results, "apps": apps_block}
         print(json.dumps(out), flush=True)
     ctx.close()
 

@@ -44,6 +44,8 @@ class Micro:
         init = torch.from_numpy(init_np.astype(np.int32)).to(dev)
         if variant in ("cuda", "typeptr_heap"):
             self.objs = ctx.alloc_cuda(vf.APP_MICRO, self.types, init, tag=(variant == "typeptr_heap"))
+        elif variant == "cuda_packed":
+            self.objs = ctx.alloc_packed(vf.APP_MICRO, self.types, init)
         else:
             self.objs = ctx.alloc_typed_batch(vf.APP_MICRO, self.types, init, tag=(variant == "typeptr"))
         torch.cuda.synchronize(dev)

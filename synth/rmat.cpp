@@ -17,6 +17,7 @@
 #include <vector>
 #ifdef _OPENMP
 #include <omp.h>
+#include <parallel/algorithm>
 #endif
 
 static inline uint64_t splitmix64(uint64_t x) {
@@ -60,9 +61,13 @@ void synth_permutation(uint64_t n, uint64_t seed, uint64_t stream, uint32_t* per
     key[v] = draw(seed, stream, (uint64_t)v);
     idx[v] = (uint32_t)v;
   }
-  std::sort(idx.begin(), idx.end(), [&](uint32_t a, uint32_t b) {
-    return key[a] < key[b] || (key[a] == key[b] && a < b);
-  });
+  // (key, index) pairs are distinct: any correct sort gives the same order
+  auto less = [&](uint32_t a, uint32_t b) { return key[a] < key[b] || (key[a] == key[b] && a < b); };
+#ifdef _OPENMP
+  __gnu_parallel::sort(idx.begin(), idx.end(), less);
+#else
+  std::sort(idx.begin(), idx.end(), less);
+#endif
   for (uint64_t r = 0; r < n; ++r) perm[idx[r]] = (uint32_t)r;
 }
 
@@ -71,22 +76,26 @@ void synth_permutation(uint64_t n, uint64_t seed, uint64_t stream, uint32_t* per
 // Fills offs[0..V] and col (capacity >= 2*nedges); returns the arc count.
 uint64_t synth_csr(uint64_t V, uint64_t nedges, const uint32_t* src, const uint32_t* dst,
                    const uint32_t* perm, uint64_t* offs, uint32_t* col) {
-  // raw degree with duplicates
+  // raw degree with duplicates (parallel; counts are order-free)
   std::vector<uint64_t> rawdeg(V + 1, 0);
-  for (uint64_t e = 0; e < nedges; ++e) {
+#pragma omp parallel for schedule(static)
+  for (int64_t e = 0; e < (int64_t)nedges; ++e) {
     uint32_t s = perm ? perm[src[e]] : src[e], d = perm ? perm[dst[e]] : dst[e];
     if (s == d) continue;
-    ++rawdeg[s + 1];
-    ++rawdeg[d + 1];
+    __atomic_fetch_add(&rawdeg[s + 1], 1ull, __ATOMIC_RELAXED);
+    __atomic_fetch_add(&rawdeg[d + 1], 1ull, __ATOMIC_RELAXED);
   }
   for (uint64_t v = 0; v < V; ++v) rawdeg[v + 1] += rawdeg[v];
   std::vector<uint32_t> adj(rawdeg[V]);
   std::vector<uint64_t> fill(rawdeg.begin(), rawdeg.end() - 1);
-  for (uint64_t e = 0; e < nedges; ++e) {
+  // scatter in parallel: the order inside a list is arbitrary here, but every
+  // list is sorted and de-duplicated below, so the CSR is deterministic
+#pragma omp parallel for schedule(static)
+  for (int64_t e = 0; e < (int64_t)nedges; ++e) {
     uint32_t s = perm ? perm[src[e]] : src[e], d = perm ? perm[dst[e]] : dst[e];
     if (s == d) continue;
-    adj[fill[s]++] = d;
-    adj[fill[d]++] = s;
+    adj[__atomic_fetch_add(&fill[s], 1ull, __ATOMIC_RELAXED)] = d;
+    adj[__atomic_fetch_add(&fill[d], 1ull, __ATOMIC_RELAXED)] = s;
   }
   std::vector<uint64_t> udeg(V, 0);
 #pragma omp parallel for schedule(dynamic, 4096)

@@ -79,3 +79,28 @@ def test_gen_threads_identical():
     b = oracle.gen_run(W, H, s0, 20, threads=oracle.max_threads())
     for x, y in zip(a[:3], b[:3]):
         assert np.array_equal(x, y)
+
+
+@pytest.mark.parametrize("rule", [("2", "345", 4), ("34", "34", 6), ("3", "23", 2)])
+def test_gen_counters_definition(rule):
+    """The counter of a cell's current object (Dead / Alive / Dying; each next()
+    call increments it, a type change swaps in the other object with counter 0,
+    P:1530-1534 reading G15) = generations since the cell's KIND last changed,
+    derived here from the textbook state sequence (all dying states 2..C-1 are
+    one kind: the Dying object just advances its stage)."""
+    born, surv, C = rule
+    W, H, G = 27, 19, 30
+    s0 = synth.soup(W, H, seed=12)
+    seq = [s0.reshape(H, W).astype(np.int32)] + textbook_generations(s0.reshape(H, W), G, born, surv, C)
+    kind = [np.minimum(s, 2) for s in seq]
+    _, ctr, _, _ = oracle.gen_run(W, H, s0, G, born, surv, C)
+    c2 = ctr.reshape(H, W)
+    changed = 0
+    for y in range(H):
+        for x in range(W):
+            k = 0
+            while k < G and kind[G - k][y, x] == kind[G - k - 1][y, x]:
+                k += 1
+            assert c2[y, x] == k
+            changed += k < G
+    assert 0 < changed < W * H  # both branches of the derivation are exercised
