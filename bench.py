@@ -44,7 +44,7 @@ def parse():
     ap.add_argument("--variant", default="typeptr", choices=["cuda", "sharedoa", "coal", "typeptr"])
     ap.add_argument("--T", type=int, default=4)
     ap.add_argument("--order", default="random", choices=["random", "sorted", "kperwarp"])
-    ap.add_argument("--n", type=int, default=1 << 26)
+    ap.add_argument("--n", "--objects", dest="n", type=int, default=1 << 26)
     ap.add_argument("--seed", type=int, default=42)
     ap.add_argument("--cuda-n", type=int, default=1 << 24,
                     help="objects for the same-config comparison with the device-heap CUDA baseline (device "
@@ -52,6 +52,10 @@ def parse():
     ap.add_argument("--apps", default=",".join(("gol", "ray", "nbody", "gen", "traf", "stut", "collide", "graph")),
                     help="per-app block (BASELINE configs 1, 3, 4, 5); '' to skip")
     ap.add_argument("--app-variants", default="cuda,cuda_packed,sharedoa,coal,typeptr")
+    ap.add_argument("--app-small", action="store_true",
+                    help="per-app block at code-path test sizes (tests only; not a BASELINE config)")
+    ap.add_argument("--strong", action="store_true",
+                    help="N > 1: split ONE array of --n objects into contiguous blocks (default: weak, --n per GPU)")
     ap.add_argument("--no-variants", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
@@ -111,6 +115,14 @@ class Clocks:
 
 
 # --------------------------------------------------------------------------- helpers
+def max_over_ranks(ms, dev):
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor([ms], dtype=torch.float64, device="cpu" if dist.get_backend() == "gloo" else dev)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
 def peaks():
     try:
         return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
@@ -160,12 +172,14 @@ def oracle_micro_sample(args, n_s, reps, threads):
 def workload_config(args, world):
     """The workload both arms measure (the reference arm times a bounded sample
     of it on the host; its cpu_baseline.sample says which)."""
-    return {"workload": f"micro: n={args.n} objects/GPU x T={args.T} types, {args.order} order, "
+    strong = getattr(args, "strong", False) and world > 1
+    per = f"{args.n} objects in total, contiguous blocks of n/{world} per GPU" if strong else f"{args.n} objects/GPU"
+    return {"workload": f"micro: n={per} x T={args.T} types, {args.order} order, "
                         f"1 virtual apply() per object per step",
             "variant": args.variant, "n": args.n, "T": args.T, "order": args.order,
             "seed": args.seed, "object_bytes": 16,
             "l2": "inputs larger than L2 (1.5 GiB objects+pointers per GPU >> 126 MB)",
-            "parallelism": f"dp{world} (independent object shards)"}
+            "parallelism": f"dp{world} ({'strong: one array split into index blocks' if strong else 'weak: independent object shards'})"}
 
 
 def run_reference(args, rank, world):
@@ -206,9 +220,19 @@ def run_ours(args, rank, world, local):
     dev = torch.device(f"cuda:{local}")
     ctx = vf.Ctx(local, cuda_heap_bytes=16 << 30)
     s = torch.cuda.Stream(device=dev)
-    n = args.n
-    types = synth.micro_types(n, args.T, args.order, seed=args.seed + rank)
-    init = synth.micro_init(n, seed=args.seed + rank)
+    if args.strong and world > 1:
+        # strong scaling: ONE array of args.n objects, contiguous
+        # index blocks of n / world per rank (same global draws as N = 1)
+        per = -(-args.n // world)
+        lo, hi = min(args.n, rank * per), min(args.n, (rank + 1) * per)
+        types = synth.micro_types(args.n, args.T, args.order, seed=args.seed)[lo:hi].copy()
+        init = synth.micro_init(args.n, seed=args.seed)[lo:hi].copy()
+        n = hi - lo
+    else:
+        n = args.n
+        types = synth.micro_types(n, args.T, args.order, seed=args.seed + rank)
+        init = synth.micro_init(n, seed=args.seed + rank)
+    n_total = args.n if (args.strong and world > 1) else world * n
 
     def barrier():
         if world > 1:
@@ -232,9 +256,7 @@ def run_ours(args, rank, world, local):
         launches = vf.launch_count() - l0
         ms = e0.elapsed_time(e1)
         if world > 1:
-            t = torch.tensor([ms], device=dev)
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            ms = float(t.item())
+            ms = max_over_ranks(ms, dev)
         return ms, launches
 
     flush_buf = None
@@ -268,7 +290,7 @@ def run_ours(args, rank, world, local):
     ms, launches = timed(m, args.steps, args.warmup)
     clk = clocks.stop()
     step_ms = ms / args.steps
-    value = world * n * args.steps / (ms / 1e3)
+    value = n_total * args.steps / (ms / 1e3)
     # parity spot-check of the timed objects (closed form on a sample; oracle parity lives in tests/)
     reps = args.warmup + args.steps
     vals = m.values().cpu().numpy()
@@ -308,10 +330,8 @@ def run_ours(args, rank, world, local):
         torch.cuda.synchronize(dev)
         e_ms = e0.elapsed_time(e1)
         if world > 1:
-            t = torch.tensor([e_ms], device=dev)
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            e_ms = float(t.item())
-        e2e = {"value": world * n * e2e_steps / (e_ms / 1e3), "unit": "calls/s",
+            e_ms = max_over_ranks(e_ms, dev)
+        e2e = {"value": n_total * e2e_steps / (e_ms / 1e3), "unit": "calls/s",
                "h2d_bytes_per_step": 8 * n, "d2h_bytes_per_step": 8,
                "path": "pinned host pointer array -> vf_dispatch_host(apply; chunked H2D overlapped with the "
                        "calls) -> vf_dispatch(get) -> vf_checksum_i32 -> 8 B D2H"}
@@ -327,7 +347,7 @@ def run_ours(args, rank, world, local):
                 continue
             mv = apps.Micro(ctx, n, args.T, variant=variant, types_np=types, init_np=init)
             vms, _ = timed(mv, max(20, args.steps // 4), args.warmup)
-            results[variant] = {"calls_per_s": world * n * max(20, args.steps // 4) / (vms / 1e3), "n": n}
+            results[variant] = {"calls_per_s": n_total * max(20, args.steps // 4) / (vms / 1e3), "n": n}
             del mv
             ctx.reset()
         # device-heap `new` baseline (paper's CUDA) at a size it allocates in seconds
@@ -376,7 +396,7 @@ def run_ours(args, rank, world, local):
 
         apps_block = apps_bench.run_apps(env, names, tuple(args.app_variants.split(",")),
                                          cpu=(rank == 0 and world == 1 and not args.no_cpu), clocks_cls=Clocks,
-                                         log=log)
+                                         log=log, small=args.app_small)
 
     pk = peaks()
     hbm = pk.get("hbm_gbs")
@@ -399,7 +419,8 @@ def run_ours(args, rank, world, local):
     if rank == 0:
         out = {"metric": "virtual calls/s (config 2 dispatch microbenchmark)", "value": value,
                "unit": "calls/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
-               "ms_per_step": step_ms, "higher_is_better": True, "scaling": "weak",
+               "ms_per_step": step_ms, "higher_is_better": True,
+               "scaling": "strong" if (args.strong and world > 1) else "weak",
                "vs_baseline": None, "dtype": "int32", "data": "synthetic",
                "config": workload_config(args, world),
                "gpu_launches": launches, "parity_sample_ok": ok, "roofline": roof, "clocks": clk,
@@ -413,10 +434,14 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    # test hooks (tests/test_gpu_bench_multirank.py): run N ranks on ONE GPU over
+    # gloo (NCCL refuses two ranks on one device); never set by the driver
+    if os.environ.get("VF_BENCH_DEVICE") is not None:
+        local = int(os.environ["VF_BENCH_DEVICE"])
     if world > 1:
         import torch.distributed as dist
-        backend = "gloo" if args.impl == "reference" else "nccl"
-        if backend == "nccl":
+        backend = "gloo" if args.impl == "reference" else os.environ.get("VF_BENCH_BACKEND", "nccl")
+        if args.impl != "reference":
             import torch
             torch.cuda.set_device(local)
         dist.init_process_group(backend)

@@ -720,7 +720,10 @@ vf_status vf_checksum_i32(const int32_t* vals_dev, uint64_t n, long long* out_de
  * grids of <= 2^17 cells in ONE thread-block cluster (state in distributed
  * shared memory, hardware cluster barrier), 0 (default; measured faster on
  * B200: a 16-SM cluster serialises 4 cells per thread) always uses the
- * cooperative grid-barrier kernel.
+ * cooperative grid-barrier kernel; "ray_minblocks" = 4 (default) or 5: the
+ * ray tracer's direct kernel compiled for >= that many resident CTAs per SM.
+ * The unroll / prefetch / pipeline knobs apply to config 2's app (micro);
+ * the other apps run their default launch configuration.
  * VF_ERR_INVALID for unknown keys / values. */
 vf_status vf_set_tuning(const char* key, int value);
 /* Number of libvf kernel launches issued since load (for bench accounting). */

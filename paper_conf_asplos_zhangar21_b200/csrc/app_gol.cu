@@ -233,7 +233,7 @@ __global__ void __launch_bounds__(kBlock) k_run_grouped(RunArgs r, DevTable tbl)
         r.nbr[c] = count_live_cg(r.W, r.H, r.torus, prev, c);
         p = r.grid[c];
       }
-      if (p) t = R::resolve(smem, tbl.P, p, ad, hint);
+      if (p) t = R::resolve(smem, tbl, p, ad, hint);
       group_call<App, VF_GOL_NEXT>(t, ad, p, c, args, tbl);
       if (valid) post_cg(r, prev, next, c);
     }
@@ -326,7 +326,7 @@ __global__ void __launch_bounds__(kClusterBlock, 1) k_run_cluster(RunArgs r, Dev
         prev_s = cur[k];
         p = r.grid[c];
       }
-      if (p) t = R::resolve(smem, tbl.P, p, ad, hint);
+      if (p) t = R::resolve(smem, tbl, p, ad, hint);
       group_call<App, VF_GOL_NEXT>(t, ad, p, c, args, tbl);
       if (valid) {
         const uint8_t s = *(volatile const uint8_t*)(next + c);  // this thread's own write

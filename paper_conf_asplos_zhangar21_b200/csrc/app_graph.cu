@@ -43,16 +43,20 @@ struct VertexK final : Vertex {
 
   __device__ void bfs_expand(vf_graph_bfs_args a, uint64_t i) {
     const Work w = work_of(a.offs_dev, a.chunk_dev, i, vid, deg, a.C);
+    const uint64_t keep = l2_keep();
     for_neighbors<U>(a.col_dev, w.b, w.e, [&](uint32_t u) {
-      if (a.depth_dev[u] == -1 && atomicCAS(a.depth_dev + u, -1, a.level + 1) == -1) enqueue(a, u);
+      if (ld_hint_rw(a.depth_dev + u, keep) == -1 && atomicCAS(a.depth_dev + u, -1, a.level + 1) == -1) enqueue(a, u);
     });
   }
   // bottom-up step: an unvisited vertex joins level+1 if a neighbour is at `level`
   __device__ void bfs_probe(vf_graph_bfs_args a, uint64_t i) {
     if (*(volatile int32_t*)(a.depth_dev + vid) != -1) return;
     const Work w = work_of(a.offs_dev, a.chunk_dev, i, vid, deg, a.C);
+    const uint64_t keep = l2_keep();
     for (uint64_t k = w.b; k < w.e; ++k) {
-      if (a.depth_dev[__ldg(a.col_dev + k)] == a.level) {
+      // depth values of earlier levels are final: a stale read of this
+      // launch's updates (level + 1) cannot equal `level`
+      if (ld_hint(a.depth_dev + __ldg(a.col_dev + k), keep) == a.level) {
         if (atomicCAS(a.depth_dev + vid, -1, a.level + 1) == -1) *(volatile uint32_t*)a.next_count_dev = 1u;
         return;
       }
@@ -62,9 +66,10 @@ struct VertexK final : Vertex {
   __device__ void bfs_probe_bits(vf_graph_bfs_bits_args a, uint64_t i) {
     if (*(volatile int32_t*)(a.depth_dev + vid) != -1) return;
     const Work w = work_of(a.offs_dev, a.chunk_dev, i, vid, deg, a.C);
+    const uint64_t keep = l2_keep();
     for (uint64_t k = w.b; k < w.e; ++k) {
       const uint32_t u = __ldg(a.col_dev + k);
-      if ((__ldg(a.frontier_dev + (u >> 5)) >> (u & 31u)) & 1u) {
+      if ((ld_hint(a.frontier_dev + (u >> 5), keep) >> (u & 31u)) & 1u) {
         if (atomicCAS(a.depth_dev + vid, -1, a.level + 1) == -1) {
           atomicOr(a.next_dev + (vid >> 5), 1u << (vid & 31u));
           *(volatile uint32_t*)a.next_count_dev = 1u;
@@ -76,9 +81,10 @@ struct VertexK final : Vertex {
   __device__ void cc_update(vf_graph_cc_args a, uint64_t i) {
     const Work w = work_of(a.offs_dev, a.chunk_dev, i, vid, deg, a.C);
     const uint32_t own = __ldg(a.label_in_dev + vid);
+    const uint64_t keep = l2_keep();
     uint32_t m = own;
     if constexpr (U == 1) {
-      for_neighbors<1>(a.col_dev, w.b, w.e, [&](uint32_t u) { m = min(m, __ldg(a.label_in_dev + u)); });
+      for_neighbors<1>(a.col_dev, w.b, w.e, [&](uint32_t u) { m = min(m, ld_hint(a.label_in_dev + u, keep)); });
     } else {
       uint32_t acc[U];
 #pragma unroll
@@ -86,9 +92,9 @@ struct VertexK final : Vertex {
       uint64_t k = w.b;
       for (; k + U <= w.e; k += U) {
 #pragma unroll
-        for (int j = 0; j < U; ++j) acc[j] = min(acc[j], __ldg(a.label_in_dev + __ldg(a.col_dev + k + j)));
+        for (int j = 0; j < U; ++j) acc[j] = min(acc[j], ld_hint(a.label_in_dev + __ldg(a.col_dev + k + j), keep));
       }
-      for (; k < w.e; ++k) acc[0] = min(acc[0], __ldg(a.label_in_dev + __ldg(a.col_dev + k)));
+      for (; k < w.e; ++k) acc[0] = min(acc[0], ld_hint(a.label_in_dev + __ldg(a.col_dev + k), keep));
 #pragma unroll
       for (int j = 0; j < U; ++j) m = min(m, acc[j]);
     }
@@ -113,10 +119,11 @@ struct VertexK final : Vertex {
   }
   __device__ void pr_update(vf_graph_pr_args a, uint64_t i) {
     const Work w = work_of(a.offs_dev, a.chunk_dev, i, vid, deg, a.C);
+    const uint64_t keep = l2_keep();
     double s;
     if constexpr (U == 1) {
       s = 0.0;
-      for_neighbors<1>(a.col_dev, w.b, w.e, [&](uint32_t u) { s += __ldg(a.contrib_dev + u); });
+      for_neighbors<1>(a.col_dev, w.b, w.e, [&](uint32_t u) { s += ld_hint(a.contrib_dev + u, keep); });
     } else {
       double acc[U];
 #pragma unroll
@@ -124,9 +131,9 @@ struct VertexK final : Vertex {
       uint64_t k = w.b;
       for (; k + U <= w.e; k += U) {
 #pragma unroll
-        for (int j = 0; j < U; ++j) acc[j] += __ldg(a.contrib_dev + __ldg(a.col_dev + k + j));
+        for (int j = 0; j < U; ++j) acc[j] += ld_hint(a.contrib_dev + __ldg(a.col_dev + k + j), keep);
       }
-      for (; k < w.e; ++k) acc[0] += __ldg(a.contrib_dev + __ldg(a.col_dev + k));
+      for (; k < w.e; ++k) acc[0] += ld_hint(a.contrib_dev + __ldg(a.col_dev + k), keep);
       s = 0.0;
 #pragma unroll
       for (int j = 0; j < U; ++j) s += acc[j];

@@ -384,6 +384,12 @@ DevTable dev_table(vf_ctx* c, uint32_t app) {
   d.ntypes = app_ops(app)->ntypes;
   d.active_types = 0;
   for (uint64_t k : c->type_count[app]) d.active_types += (k != 0);
+  for (uint32_t j = 0; j < kTableInline; ++j) {
+    const bool v = j < t.K && t.K <= kTableInline;
+    d.in_start[j] = v ? t.rows[j].start : ~0ull;
+    d.in_end[j] = v ? t.rows[j].end : 0ull;
+    d.in_type[j] = v ? t.rows[j].type_id : VF_NOT_FOUND;
+  }
   return d;
 }
 
@@ -451,6 +457,9 @@ vf_status vf_set_tuning(const char* key, int value) {
   } else if (!strcmp(key, "cluster")) {
     if (value < 0 || value > 1) return VF_ERR_INVALID;
     tuning().cluster = value;
+  } else if (!strcmp(key, "ray_minblocks")) {
+    if (value != 4 && value != 5) return VF_ERR_INVALID;
+    tuning().ray_minblocks = value;
   } else {
     return VF_ERR_INVALID;
   }

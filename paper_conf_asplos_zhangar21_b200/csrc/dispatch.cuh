@@ -85,22 +85,28 @@ __device__ __forceinline__ void prefetch_l1(uint64_t a) {
 struct ResolveTP {
   static constexpr bool kNeedsTable = false;
   __device__ static void stage(unsigned char*, const DevTable&) {}
-  __device__ __forceinline__ static uint32_t resolve(const unsigned char*, uint32_t,
-                                                     uint64_t p, uint64_t& a, uint32_t&) {
+  __device__ __forceinline__ static uint32_t resolve(const unsigned char*, const DevTable&, uint64_t p, uint64_t& a,
+                                                     uint32_t&) {
     a = strip(p);
     const uint32_t tag = (uint32_t)(p >> 32) >> (VF_VA_BITS - 32);
     return tag - 1u;  // tag 0 (untagged) -> 0xFFFFFFFF = not found -> fallback
   }
 };
 
-// COAL (§5, Algorithm 1): the virtual range table is staged into
-// shared memory once per CTA and searched per lane. The segment tree of
-// P:1158-1174 answers "which disjoint [start,end) contains p"; over sorted
-// disjoint ranges that is exactly "the last start <= p, then p < end", which
-// we do as a branch-free binary search (log2 P dependent LDS + SEL).
+// COAL (§5, Algorithm 1): the segment tree of P:1158-1174 answers
+// "which disjoint [start,end) contains p"; over sorted disjoint ranges that is
+// exactly "the last start <= p, then p < end".
+//  * K <= kTableInline rows (every app here with its VA windows: K = #types):
+//    the table rides in the kernel parameters (constant bank) and each lane
+//    tests the K ranges directly against constant operands — no shared-memory
+//    staging, no CTA barrier, no dependent load;
+//  * larger tables (config 2 at T = 32, fragmented K): staged into shared
+//    memory once per CTA and searched per lane branch-free (log2 P dependent
+//    LDS + SEL, then the end check).
 struct ResolveCOAL {
   static constexpr bool kNeedsTable = true;
   __device__ static void stage(unsigned char* smem, const DevTable& t) {
+    if (t.K <= kTableInline) return;  // searched in the parameter bank (CTA-uniform)
     uint64_t* s_start = reinterpret_cast<uint64_t*>(smem);
     uint64_t* s_end = s_start + t.P;
     uint32_t* s_type = reinterpret_cast<uint32_t*>(s_end + t.P);
@@ -112,18 +118,27 @@ struct ResolveCOAL {
     }
     __syncthreads();
   }
-  // Always the full branch-free search (log2 P dependent LDS.64 + SEL, then
-  // the end check): measured on B200 faster than first testing the lane's
-  // previous range (config 2, T = 4: 129.8 -> 133.4 Gcalls/s), since with
-  // mixed types the test mostly misses and splits the warp. `hint` is unused.
-  __device__ __forceinline__ static uint32_t resolve(const unsigned char* smem, uint32_t P,
-                                                     uint64_t p, uint64_t& a, uint32_t& hint) {
-    const uint64_t* s_start = reinterpret_cast<const uint64_t*>(smem);
-    const uint64_t* s_end = s_start + P;
-    const uint32_t* s_type = reinterpret_cast<const uint32_t*>(s_end + P);
+  // Always the full search (measured on B200 faster than first testing the
+  // lane's previous range: with mixed types the test mostly misses and splits
+  // the warp). `hint` is unused.
+  __device__ __forceinline__ static uint32_t resolve(const unsigned char* smem, const DevTable& tbl, uint64_t p,
+                                                     uint64_t& a, uint32_t& hint) {
     a = strip(p);  // a TypePointer-tagged pointer is searched (and dereferenced) by its address
     p = a;
     (void)hint;
+    if (tbl.K <= kTableInline) {
+      uint32_t t = kNF;
+#pragma unroll
+      for (uint32_t j = 0; j < kTableInline; ++j) {
+        if (j >= tbl.K) break;  // uniform
+        t = (p >= tbl.in_start[j] && p < tbl.in_end[j]) ? tbl.in_type[j] : t;
+      }
+      return t;
+    }
+    const uint32_t P = tbl.P;
+    const uint64_t* s_start = reinterpret_cast<const uint64_t*>(smem);
+    const uint64_t* s_end = s_start + P;
+    const uint32_t* s_type = reinterpret_cast<const uint32_t*>(s_end + P);
     uint32_t j = 0;
     for (uint32_t step = P >> 1; step > 0; step >>= 1) {
       const uint32_t c = j + step;
@@ -233,7 +248,7 @@ __global__ void __launch_bounds__(kBlock, MinBlocks<App>::value) k_dispatch_grou
     uint32_t t[U];
 #pragma unroll
     for (int j = 0; j < U; ++j) {
-      t[j] = p[j] ? R::resolve(smem, tbl.P, p[j], a[j], hint) : kNF;
+      t[j] = p[j] ? R::resolve(smem, tbl, p[j], a[j], hint) : kNF;
       if (!p[j]) a[j] = 0;
     }
     // Issue every lane's object line before the (serialised) type groups run,
@@ -257,7 +272,8 @@ __global__ void __launch_bounds__(kBlock, MinBlocks<App>::value) k_dispatch_grou
 }
 
 // ---------------------------------------------------------------------------
-// TMA-pipelined grouped dispatch (default for COAL / TypePointer).
+// TMA-pipelined grouped dispatch (tuning key "pipeline" = 1; measured slower
+// than the type-sorted kernel below, which is the default).
 //
 // The pointer array is a pure stream: one elected thread per CTA moves each
 // tile of kBlock*U pointers global -> shared with cp.async.bulk (TMA, 1-D)
@@ -311,12 +327,12 @@ struct PipeSmem {
 // values are returned in w[] and folded into `sink` only when the tile becomes
 // current, so the wait for them overlaps the previous tile's group walk.
 template <class App, int M, class R, int U, int PF>
-__device__ __forceinline__ void resolve_tile(const unsigned char* smem, uint32_t P, const uint64_t (&p)[U],
+__device__ __forceinline__ void resolve_tile(const unsigned char* smem, const DevTable& tbl, const uint64_t (&p)[U],
                                              uint64_t (&a)[U], uint32_t (&t)[U], uint32_t (&w)[U],
                                              uint32_t& hint) {
 #pragma unroll
   for (int j = 0; j < U; ++j) {
-    t[j] = p[j] ? R::resolve(smem, P, p[j], a[j], hint) : kNF;
+    t[j] = p[j] ? R::resolve(smem, tbl, p[j], a[j], hint) : kNF;
     if (!p[j]) a[j] = 0;
     w[j] = 0;
   }
@@ -379,7 +395,7 @@ __global__ void __launch_bounds__(kBlock, 4) k_dispatch_pipe(const uint64_t* __r
       mbar_expect_tx(&bars[s], WT * sizeof(uint64_t));
       tma_load_1d(ring + (size_t)s * WT, objs + tile_base(k + S), WT * sizeof(uint64_t), &bars[s]);
     }
-    resolve_tile<App, M, R, U, PF>(smem, tbl.P, p, a, t, w, hint);
+    resolve_tile<App, M, R, U, PF>(smem, tbl, p, a, t, w, hint);
   };
 
   if (has(0)) fetch(0, pc, ac, tc, wc);
@@ -408,7 +424,7 @@ __global__ void __launch_bounds__(kBlock, 4) k_dispatch_pipe(const uint64_t* __r
       const uint64_t idx = base + (uint64_t)j * 32 + lane;
       pc[j] = idx < n ? ldg_u64(objs + idx) : 0ull;
     }
-    resolve_tile<App, M, R, U, PF>(smem, tbl.P, pc, ac, tc, wc, hint);
+    resolve_tile<App, M, R, U, PF>(smem, tbl, pc, ac, tc, wc, hint);
 #pragma unroll
     for (int j = 0; j < U; ++j) {
       sink ^= wc[j];
@@ -495,7 +511,7 @@ __global__ void __launch_bounds__(kBlock, MinBlocks<App>::value) k_dispatch_sort
     }
 #pragma unroll
     for (int j = 0; j < U; ++j) {
-      t[j] = p[j] ? R::resolve(smem, tbl.P, p[j], a[j], hint) : kNF;
+      t[j] = p[j] ? R::resolve(smem, tbl, p[j], a[j], hint) : kNF;
       if (!p[j]) a[j] = 0;
       const bool fb = t[j] >= (uint32_t)App::kTypes && p[j] != 0;
       if (__any_sync(0xffffffffu, fb)) {
@@ -682,7 +698,7 @@ __global__ void __launch_bounds__(kBlock, MinBlocks<App>::value) k_dispatch_indi
     const uint64_t p = ldg_u64(objs + i);
     if (!p) continue;
     uint64_t a;
-    const uint32_t t = R::resolve(smem, tbl.P, p, a, hint);
+    const uint32_t t = R::resolve(smem, tbl, p, a, hint);
     if (t < (uint32_t)App::kTypes) {
       const ThunkFn f = s_fn[t];  // vFunc* = table[type]
       f(a, i, &s_args);           // indirect CALL
@@ -752,8 +768,8 @@ __device__ __forceinline__ uint32_t resolve_rule(int variant, const unsigned cha
   if (!p) return kNF;
   uint64_t a;
   uint32_t hint = 0;
-  if (variant == VF_TYPEPTR) return ResolveTP::resolve(smem, tbl.P, p, a, hint);
-  if (variant == VF_COAL) return ResolveCOAL::resolve(smem, tbl.P, p, a, hint);
+  if (variant == VF_TYPEPTR) return ResolveTP::resolve(smem, tbl, p, a, hint);
+  if (variant == VF_COAL) return ResolveCOAL::resolve(smem, tbl, p, a, hint);
   if (variant == VF_CONCORD) {
     if constexpr (TagOffset<App>::value >= 0) {
       const uint32_t t = *reinterpret_cast<const uint32_t*>(strip(p) + TagOffset<App>::value);
@@ -1142,7 +1158,7 @@ __global__ void __launch_bounds__(kBlock) k_step_grouped(uint64_t n, ArgBlob arg
       st.pre(c);
       p = st.ptr(c);
     }
-    if (p) t = R::resolve(smem, tbl.P, p, a, hint);
+    if (p) t = R::resolve(smem, tbl, p, a, hint);
     if constexpr (HasWarm<Step>::value) {
       uint32_t sink = 0;
       if (valid && t < (uint32_t)App::kTypes) sink = st.warm(c, a);

@@ -7,6 +7,45 @@
 namespace vf {
 namespace graph {
 
+// L2 residency (B200: 126 MB of L2). The per-vertex state a body gathers at
+// random (PageRank contributions, CC labels, BFS depths / frontier bits: 64-
+// 134 MB at RMAT-24) is loaded with an evict_last policy so the adjacency
+// stream `col` (2 GB, read once per sweep) does not push it out of L2. (An
+// evict_first policy on `col` itself was measured worse on B200: a lane reads
+// its row 4 B at a time, and the sector was evicted between its reads.)
+__device__ __forceinline__ uint64_t l2_keep() {
+  uint64_t p;
+  asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ uint64_t l2_stream() {
+  uint64_t p;
+  asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ uint32_t ld_hint(const uint32_t* a, uint64_t pol) {
+  uint32_t v;
+  asm("ld.global.nc.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(v) : "l"(a), "l"(pol));
+  return v;
+}
+__device__ __forceinline__ int32_t ld_hint(const int32_t* a, uint64_t pol) {
+  int32_t v;
+  asm("ld.global.nc.L2::cache_hint.s32 %0, [%1], %2;" : "=r"(v) : "l"(a), "l"(pol));
+  return v;
+}
+__device__ __forceinline__ double ld_hint(const double* a, uint64_t pol) {
+  double v;
+  asm("ld.global.nc.L2::cache_hint.f64 %0, [%1], %2;" : "=d"(v) : "l"(a), "l"(pol));
+  return v;
+}
+
+// coherent (non-.nc) load with a policy: state this kernel also writes
+__device__ __forceinline__ int32_t ld_hint_rw(const int32_t* a, uint64_t pol) {
+  int32_t v;
+  asm volatile("ld.global.L2::cache_hint.s32 %0, [%1], %2;" : "=r"(v) : "l"(a), "l"(pol));
+  return v;
+}
+
 // Neighbour loop with U independent lanes of work (U = 1: plain loop).
 template <int U, class F>
 __device__ __forceinline__ void for_neighbors(const uint32_t* __restrict__ col, uint64_t b, uint64_t e, F&& f) {

@@ -20,6 +20,11 @@ struct __align__(16) ArgBlob {
 };
 
 // Device view of one app's virtual range table (sorted, merged) and vTables.
+// Tables of <= kTableInline rows also travel inline in the kernel parameters
+// (constant bank), so a COAL CTA stages them into shared memory without a
+// dependent global load at its start (the paper keeps the table in
+// constant / shared memory).
+constexpr uint32_t kTableInline = 8;
 struct DevTable {
   const uint64_t* start;  // K entries, sorted
   const uint64_t* end;    // K entries
@@ -29,6 +34,9 @@ struct DevTable {
   const uint64_t* vptr;   // ntypes entries: device vTable* per concrete type
   uint32_t ntypes;
   uint32_t active_types;  // concrete types with live objects (launch heuristics)
+  uint64_t in_start[kTableInline];  // rows 0..K-1 when K <= kTableInline
+  uint64_t in_end[kTableInline];
+  uint32_t in_type[kTableInline];
 };
 
 struct AppOps {
@@ -114,6 +122,7 @@ struct Tuning {
   int call = 0;       // COAL / TypePointer: 0 grouped direct call, 1 indirect CALL via vFunc* table
   int persistent = -1; // grouped kernels: 1 persistent grid, 0 one tile per CTA, -1 app default (kHeavyMask)
   int cluster = 0;     // vf_gol_run: 1 one thread-block cluster (state in DSMEM) when the grid fits
+  int ray_minblocks = 4;  // k_ray_direct __launch_bounds__ min CTAs per SM (4: <= 64 regs, 5: <= 48)
 };
 Tuning& tuning();
 

@@ -70,21 +70,24 @@ class Env:
             import torch.distributed as dist
             dist.barrier(group=self.group)
 
+    def _reduce(self, x, dtype, op):
+        import torch.distributed as dist
+        dev = "cpu" if dist.get_backend(self.group) == "gloo" else self.dev
+        t = torch.tensor([x], dtype=dtype, device=dev)
+        dist.all_reduce(t, op=op, group=self.group)
+        return t.item()
+
     def max_ms(self, ms: float) -> float:
         if self.world == 1:
             return ms
         import torch.distributed as dist
-        t = torch.tensor([ms], device=self.dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX, group=self.group)
-        return float(t.item())
+        return float(self._reduce(ms, torch.float64, dist.ReduceOp.MAX))
 
     def sum_i(self, x: int) -> int:
         if self.world == 1:
             return int(x)
         import torch.distributed as dist
-        t = torch.tensor([int(x)], dtype=torch.int64, device=self.dev)
-        dist.all_reduce(t, group=self.group)
-        return int(t.item())
+        return int(self._reduce(int(x), torch.int64, dist.ReduceOp.SUM))
 
     def timed(self, step, steps: int, warmup: int):
         """ms per step: CUDA events on the app stream around `steps` calls of
@@ -140,10 +143,10 @@ def _variants(env, variants, heap_ok=True):
 
 
 # ------------------------------------------------------------------ config 1: GOL
-def app_gol(env, variants, pk, cpu=True, steps=5, warmup=2):
+def app_gol(env, variants, pk, cpu=True, steps=5, warmup=2, small=False):
     from paper_conf_asplos_zhangar21_b200 import apps
-    W = H = 256
-    gens = 100
+    W = H = 64 if small else 256
+    gens = 10 if small else 100
     g0 = synth.soup(W, H, seed=42)
     row = {"config": f"{W}x{H}, {gens} generations per step (one CUDA graph of {gens} fused generations), "
                      "dead border; 2.6 MB working set: L2-resident by construction (replicas only at N > 1)",
@@ -174,9 +177,9 @@ def app_gol(env, variants, pk, cpu=True, steps=5, warmup=2):
 
 
 # ------------------------------------------------------------------ config 3: ray tracer
-def app_ray(env, variants, pk, cpu=True, steps=3, warmup=1):
+def app_ray(env, variants, pk, cpu=True, steps=3, warmup=1, small=False):
     from paper_conf_asplos_zhangar21_b200.ray import Ray
-    W, H, S = 1920, 1080, 10000
+    W, H, S = (192, 108, 500) if small else (1920, 1080, 10000)
     types, P = synth.ray_scene(S, seed=7)
     cam = synth.ray_camera(W, H)
     tcounts = np.bincount(types, minlength=4)
@@ -209,9 +212,9 @@ def app_ray(env, variants, pk, cpu=True, steps=3, warmup=1):
 
 
 # ------------------------------------------------------------------ config 5: N-body (all pairs)
-def app_nbody(env, variants, pk, cpu=True, steps=10, warmup=3):
+def app_nbody(env, variants, pk, cpu=True, steps=10, warmup=3, small=False):
     from paper_conf_asplos_zhangar21_b200.nbody import Nbody
-    N = 65536
+    N = 2048 if small else 65536
     s = synth.nbody_system(N, seed=10)
     row = {"config": f"all-pairs N-body, N={N} bodies, 1 step (one virtual update() per body); id blocks "
                      f"over {env.world} GPU(s) + all-gather of positions; 1 MB positions L2-resident (FP32-bound)",
@@ -248,8 +251,8 @@ def _gen_once(env, v, W, s0, steps, warmup):
     return ms, st
 
 
-def app_gen(env, variants, pk, cpu=True, steps=20, warmup=3):
-    W = 4096
+def app_gen(env, variants, pk, cpu=True, steps=20, warmup=3, small=False):
+    W = 256 if small else 4096
     s0 = synth.soup(W, W, seed=42)
     row = {"config": f"{W}x{W} Generations B2/S345/C4, 1 fused generation per step; row slabs over "
                      f"{env.world} GPU(s) + halo rows; 3 x 16.8M objects (> L2)",
@@ -265,7 +268,7 @@ def app_gen(env, variants, pk, cpu=True, steps=20, warmup=3):
         row["speedup_vs_cuda_packed"] = {k: base / x["ms_per_step"] for k, x in row["variants"].items()}
     # same-config comparison with the device-heap arm (3 x 4.2M `new`s fit the bench budget)
     if "cuda" in variants and env.world == 1:
-        W2 = 2048
+        W2 = 128 if small else 2048
         s2 = synth.soup(W2, W2, seed=42)
         sub = {"config": f"{W2}x{W2} (all five variants incl. the device-heap CUDA arm; the heap arm at "
                          f"{W}x{W} needs ~6 min of device `new`)", "calls_per_step": W2 * W2, "variants": {}}
@@ -283,9 +286,9 @@ def app_gen(env, variants, pk, cpu=True, steps=20, warmup=3):
 
 
 # ------------------------------------------------------------------ config 5: TRAF
-def app_traf(env, variants, pk, cpu=True, steps=20, warmup=3):
+def app_traf(env, variants, pk, cpu=True, steps=20, warmup=3, small=False):
     from paper_conf_asplos_zhangar21_b200.traf import Traf
-    R, L = 3277, 4096
+    R, L = (37, 512) if small else (3277, 4096)
     w = synth.traf_world(R, L, seed=11)
     nveh = len(w["veh_ring"])
     row = {"config": f"{R} rings x {L} cells, {nveh} vehicles ({R * L + nveh} objects), 1 step = update() per "
@@ -311,9 +314,9 @@ def app_traf(env, variants, pk, cpu=True, steps=20, warmup=3):
 
 
 # ------------------------------------------------------------------ config 5: STUT
-def app_stut(env, variants, pk, cpu=True, steps=20, warmup=3):
+def app_stut(env, variants, pk, cpu=True, steps=20, warmup=3, small=False):
     from paper_conf_asplos_zhangar21_b200.stut import Stut
-    W = H = 2048
+    W = H = 128 if small else 2048
     w = synth.stut_lattice(W, H, seed=12, v_pull=4.0)
     n, S = W * H, len(w["a"])
     row = {"config": f"{W}x{H} nodes + {S} springs ({n + S} objects), 1 step = force() per spring + move() per "
@@ -339,9 +342,9 @@ def app_stut(env, variants, pk, cpu=True, steps=20, warmup=3):
 
 
 # ------------------------------------------------------------------ config 5: collision
-def app_collide(env, variants, pk, cpu=True, steps=5, warmup=2):
+def app_collide(env, variants, pk, cpu=True, steps=5, warmup=2, small=False):
     from paper_conf_asplos_zhangar21_b200.collide import Collide
-    N = 1 << 24
+    N = (1 << 16) if small else (1 << 24)
     s = synth.collide_system(N, seed=13)
     row = {"config": f"N={N} bodies, cutoff grid G={s['G']}, merging; 1 step = grid + update() + merge() per "
                      f"active body; id blocks over {env.world} GPU(s) + all-gathers", "variants": {}}
@@ -371,8 +374,9 @@ def app_collide(env, variants, pk, cpu=True, steps=5, warmup=2):
 
 
 # ------------------------------------------------------------------ config 4: graph
-def app_graph(env, variants, pk, cpu=True, scale=24):
+def app_graph(env, variants, pk, cpu=True, scale=24, small=False):
     from paper_conf_asplos_zhangar21_b200.graph import Graph
+    scale = 14 if small else scale
     t0 = time.time()
     offs, col = synth.rmat_graph(scale, seed=1)
     gen_s = time.time() - t0
@@ -422,7 +426,7 @@ def app_graph(env, variants, pk, cpu=True, scale=24):
     return _finish(row)
 
 
-def run_apps(env, names=ORDER, variants=ALL_VARIANTS, cpu=True, clocks_cls=None, log=None):
+def run_apps(env, names=ORDER, variants=ALL_VARIANTS, cpu=True, clocks_cls=None, log=None, small=False):
     pk = peaks()
     out = {}
     for name in names:
@@ -431,7 +435,9 @@ def run_apps(env, names=ORDER, variants=ALL_VARIANTS, cpu=True, clocks_cls=None,
         if clk:
             clk.start()
             time.sleep(0.3)
-        row = globals()[f"app_{name}"](env, variants, pk, cpu=cpu)
+        row = globals()[f"app_{name}"](env, variants, pk, cpu=cpu, small=small)
+        if small:
+            row["scale"] = "small (code-path test sizes, not a BASELINE config)"
         if clk:
             row["clocks"] = clk.stop()
         row["wall_s"] = time.time() - t0
@@ -448,12 +454,13 @@ if __name__ == "__main__":
     ap.add_argument("--variants", default=",".join(ALL_VARIANTS))
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--out", default=None)
+    ap.add_argument("--small", action="store_true", help="code-path test sizes")
     a = ap.parse_args()
     from paper_conf_asplos_zhangar21_b200 import vf
     ctx = vf.Ctx(0, cuda_heap_bytes=16 << 30)
     env = Env(ctx)
     res = run_apps(env, a.apps.split(","), tuple(a.variants.split(",")), cpu=not a.no_cpu,
-                   log=lambda n, r: print(json.dumps({n: r}), flush=True))
+                   log=lambda n, r: print(json.dumps({n: r}), flush=True), small=a.small)
     if a.out:
         json.dump(res, open(a.out, "w"), indent=1)
     ctx.close()

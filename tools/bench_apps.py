@@ -1,5 +1,7 @@
 #!/usr/bin/env python
-"""Measure every BASELINE.json config (beyond the config-2 headline in bench.py) on one B200.
+"""Round-1 per-app table (kept for GraphChi-vEN, §8f f4, and the GOL persistent forms);
+the BASELINE configs' per-app numbers now come from tools/apps_bench.py (bench.py's
+`apps` block).
 
 For each app, each dispatch variant: virtual calls/s over the timed steps
 (CUDA events on the launching stream, after warm-up), plus the algorithmic
@@ -111,14 +113,15 @@ def bench_gol(ctx, quick):
 
 # ---------------------------------------------------------------- config 5: GEN
 def bench_gen(ctx, quick):
-    W = H = 1024 if quick else 4096
+    # every variant at the same size (the device-heap arm's 3 x 16.8M `new`s at
+    # 4096^2 take ~6 min): the per-app speedups compare one config
+    W = H = 1024 if quick else 2048
     gens = 20
     s0 = synth.soup(W, H, seed=42)
     _, _, _, sec = oracle.gen_run(W, H, s0, gens, threads=oracle.max_threads())
     cpu = cpu_info(W * H * gens, sec, f"{W}x{H}, {gens} generations (same input)")
     for v in VARIANTS:
-        Wv = W if v != "cuda" else min(W, 2048)  # device-heap new of 3 x 16.8M objects takes minutes
-        sv = s0 if Wv == W else synth.soup(Wv, Wv, seed=42)
+        Wv, sv = W, s0
         g = apps.Gen(ctx, Wv, Wv, sv, v)
         ms = ev_time(g.gen, gens)
         g2 = apps.Gen(ctx, Wv, Wv, sv, v)

@@ -14,7 +14,9 @@ import sys
 sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
 from ncu_summary import raw  # noqa: E402
 
-COLS = [("duration_ns", "µs", 1e3, "{:.1f}"), ("dram_pct", "DRAM %", 1, "{:.1f}"),
+COLS = [("duration_ns", "µs", 1e3, "{:.1f}"), ("dram_gbs", "DRAM GB/s", 1, "{:.0f}"), ("dram_pct", "DRAM %", 1, "{:.1f}"),
+        ("global_ld", "global ld insts", 1, "{:.3g}"), ("branch", "branch insts", 1, "{:.3g}"),
+        ("div_targets", "divergent branch targets", 1, "{:.3g}"), ("uniform_pct", "uniform branch %", 1, "{:.1f}"),
         ("regs", "regs", 1, "{:.0f}"), ("warps_active_pct", "warps act %", 1, "{:.1f}"),
         ("simt_eff", "SIMT eff (thr/inst)", 1, "{:.1f}"), ("issue_active_pct", "issue act %", 1, "{:.1f}"),
         ("l1_hit", "L1 hit %", 1, "{:.1f}"), ("l2_hit", "L2 hit %", 1, "{:.1f}"),
@@ -36,6 +38,8 @@ def main():
         name = os.path.basename(path).replace(".raw.csv", "")
         for d in raw(path):
             traffic = d.get("dram_read", 0) + d.get("dram_write", 0)
+            if isinstance(d.get("duration_ns"), float) and d["duration_ns"] > 0:
+                d["dram_gbs"] = traffic / d["duration_ns"]
             cells = []
             for k, _, s, fmt in COLS:
                 v = d.get(k)

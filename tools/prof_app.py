@@ -78,6 +78,13 @@ def main():
         g = apps.Gen(ctx, 4096, 4096, synth.soup(4096, 4096, seed=42), a.variant)
         for _ in range(a.steps):
             g.gen()
+    elif a.app == "ray":
+        from paper_conf_asplos_zhangar21_b200.ray import Ray
+        types, P = synth.ray_scene(10000, seed=7)
+        r = Ray(ctx, types, P, a.variant)
+        cam = synth.ray_camera(1920, 1080)
+        for _ in range(a.steps):
+            r.render(1920, 1080, cam)
     elif a.app == "gol":
         g = apps.Gol(ctx, 256, 256, synth.soup(256, 256, seed=42), a.variant)
         for _ in range(a.steps):
