@@ -222,7 +222,7 @@ class Gen:
             vf.gol_neighbors(self.W, self.H, cur, self.nbr, self.torus, stream)
             self.ctx.dispatch(self.v, vf.APP_GEN, vf.GEN_NEXT, self.grid, self.args[self.parity], stream=stream)
             vf.gen_swap(self.ctx, cur, nxt, self.grid, self.dead, self.alive, self.dying, stream)
-        self.halo.exchange(nxt)
+        self.halo.exchange(nxt, stream)
         self.parity ^= 1
 
     @property

@@ -93,25 +93,25 @@ class Collide:
         self.ctx._check(self.ctx.dispatch_raw(self.v, vf.APP_COLLIDE, vf.COLLIDE_UPDATE, self.order.data_ptr(),
                                               self.n_owned, self._upd, vf._stream(stream)), "collide update")
 
-    def exchange_update(self):
+    def exchange_update(self, stream=None):
         if self.world > 1 and self.exchange:
             for b in (self._Pm, self._Vm, self._near):
-                b.gather()
+                b.gather(stream)
 
     def merge(self, stream=None):
         """Step (2): one virtual merge() per owned active body."""
         self.ctx._check(self.ctx.dispatch_raw(self.v, vf.APP_COLLIDE, vf.COLLIDE_MERGE, self.order.data_ptr(),
                                               self.n_owned, self._mrg, vf._stream(stream)), "collide merge")
 
-    def exchange_merge(self):
+    def exchange_merge(self, stream=None):
         if self.world > 1 and self.exchange:
-            self._P.gather()
+            self._P.gather(stream)
 
     def step(self, stream=None):
         self.update(stream)
-        self.exchange_update()
+        self.exchange_update(stream)
         self.merge(stream)
-        self.exchange_merge()
+        self.exchange_merge(stream)
 
     def calls(self) -> int:
         """Virtual calls issued so far by this rank (2 per owned active body per step)."""

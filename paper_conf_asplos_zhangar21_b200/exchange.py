@@ -44,6 +44,17 @@ def _staged(t: torch.Tensor, group) -> bool:
     return t.is_cuda and _dist().get_backend(group) == "gloo"
 
 
+def _on(stream, t: torch.Tensor):
+    """Run the collective (NCCL) or the staging copies (gloo) on `stream`, the
+    stream the app's kernels were enqueued on (None: the current stream)."""
+    import contextlib
+    if stream is None or not t.is_cuda:
+        return contextlib.nullcontext()
+    if not isinstance(stream, torch.cuda.Stream):
+        stream = torch.cuda.ExternalStream(int(stream), device=t.device)
+    return torch.cuda.stream(stream)
+
+
 class BlockArray:
     """Persistent padded per-id array whose owned blocks are all-gathered in place."""
 
@@ -61,10 +72,15 @@ class BlockArray:
     def data_ptr(self) -> int:
         return self.view.data_ptr()
 
-    def gather(self):
-        """After the call every rank holds every rank's block (one collective)."""
+    def gather(self, stream=None):
+        """After the call every rank holds every rank's block (one collective),
+        ordered after the work already enqueued on `stream`."""
         if self.world == 1:
             return
+        with _on(stream, self.buf):
+            self._gather()
+
+    def _gather(self):
         dist = _dist()
         if _staged(self.buf, self.group):
             if self._host is None:
@@ -79,17 +95,18 @@ class BlockArray:
             dist.all_gather_into_tensor(self.buf, self.mine, group=self.group)
 
 
-def allreduce_(t: torch.Tensor, world: int, group=None):
+def allreduce_(t: torch.Tensor, world: int, group=None, stream=None):
     """In-place sum over ranks (a few bytes: flags, the dangling mass)."""
     if world == 1:
         return
     dist = _dist()
-    if _staged(t, group):
-        h = t.cpu()
-        dist.all_reduce(h, group=group)
-        t.copy_(h)
-    else:
-        dist.all_reduce(t, group=group)
+    with _on(stream, t):
+        if _staged(t, group):
+            h = t.cpu()
+            dist.all_reduce(h, group=group)
+            t.copy_(h)
+        else:
+            dist.all_reduce(t, group=group)
 
 
 class HaloRows:
@@ -111,9 +128,13 @@ class HaloRows:
         nxt = self.rank + 1 if self.rank < self.world - 1 else (0 if self.torus else None)
         return prev, nxt
 
-    def exchange(self, state: torch.Tensor):
+    def exchange(self, state: torch.Tensor, stream=None):
         if self.world == 1 or self.r1 <= self.r0:
             return
+        with _on(stream, state):
+            self._exchange(state)
+
+    def _exchange(self, state: torch.Tensor):
         dist = _dist()
         W, H = self.W, self.H
         s2 = state.view(H, W)

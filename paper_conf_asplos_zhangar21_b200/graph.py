@@ -127,8 +127,8 @@ class Graph:
         torch.cuda.synchronize(dev)
 
     # ---------------------------------------------------------------- helpers
-    def _allreduce_sum(self, t):
-        exchange.allreduce_(t, self.world, self.group)
+    def _allreduce_sum(self, t, stream=None):
+        exchange.allreduce_(t, self.world, self.group, stream)
 
     def _dispatch(self, method, objs_ptr, n, args, stream=None):
         st = self.ctx.dispatch_raw(self.v, vf.APP_GRAPH, method, objs_ptr, n, args, vf._stream(stream))
@@ -263,13 +263,14 @@ class Graph:
 
     def pr_iteration(self, d: float = 0.85, stream=None):
         """One PageRank iteration = virtual pr_contrib() + pr_update() per owned work entry."""
-        self.dangling.zero_()
+        with exchange._on(stream, self.dangling):
+            self.dangling.zero_()
         a = vf.graph_pr_args(self.offs.data_ptr(), self.col.data_ptr(), self.rk[0].data_ptr(), self.rk[1].data_ptr(),
                              self.contrib.data_ptr(), self.dangling.data_ptr(), (1.0 - d) / self.V, d, float(self.V),
                              self.entry_chunk.data_ptr(), self.partial.data_ptr(), self.counter.data_ptr(), self.C)
         self._dispatch(vf.GRAPH_PR_CONTRIB, self.entries.data_ptr(), self.E, a, stream)
-        self._contrib.gather()
-        self._allreduce_sum(self.dangling)
+        self._contrib.gather(stream)
+        self._allreduce_sum(self.dangling, stream)
         self._dispatch(vf.GRAPH_PR_UPDATE, self.entries.data_ptr(), self.E, a, stream)
         self._rk.reverse()
         self.rk = [b.view for b in self._rk]

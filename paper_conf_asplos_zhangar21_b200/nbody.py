@@ -66,7 +66,7 @@ class Nbody:
         if st:
             self.ctx._check(st, "nbody update")
         if self.world > 1 and self.exchange:
-            self._p[1].gather()
+            self._p[1].gather(stream)
         self._p.reverse()
         self.p = [b.view for b in self._p]
 

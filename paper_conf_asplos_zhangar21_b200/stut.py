@@ -82,7 +82,7 @@ class Stut:
         if st:
             self.ctx._check(st, "stut move")
         if self.world > 1 and self.exchange:
-            self._pos.gather()
+            self._pos.gather(stream)
 
     def positions(self):
         return self.pos.cpu().numpy()
