@@ -457,9 +457,9 @@ vf_status vf_set_tuning(const char* key, int value) {
   } else if (!strcmp(key, "cluster")) {
     if (value < 0 || value > 1) return VF_ERR_INVALID;
     tuning().cluster = value;
-  } else if (!strcmp(key, "ray_minblocks")) {
-    if (value != 4 && value != 5) return VF_ERR_INVALID;
-    tuning().ray_minblocks = value;
+  } else if (!strcmp(key, "ray_rays")) {
+    if (value != 2 && value != 4) return VF_ERR_INVALID;
+    tuning().ray_rays = value;
   } else {
     return VF_ERR_INVALID;
   }

@@ -8,8 +8,8 @@ exchanged here, with NO per-call allocation:
 
 * ``BlockArray``: a per-id array that lives in a persistent buffer padded to
   ``per * world`` rows. ``view`` (the first n rows) is what the kernels index.
-  ``gather()`` is ONE ``all_gather_into_tensor`` whose input is this rank's
-  own block of the same buffer (NCCL in-place all-gather: no copy). The
+  ``gather()`` is ONE ``all_gather_into_tensor`` of this rank's block (copied
+  into a persistent send buffer, 1/world of the array) into the buffer. The
   graph's frontier bitmap, CC labels, PR contributions, N-body / STUT
   positions all use it.
 * ``HaloRows``: the GEN row slabs' halo exchange, ``batch_isend_irecv`` of
@@ -56,7 +56,7 @@ def _on(stream, t: torch.Tensor):
 
 
 class BlockArray:
-    """Persistent padded per-id array whose owned blocks are all-gathered in place."""
+    """Persistent padded per-id array whose owned blocks are all-gathered into it."""
 
     def __init__(self, n: int, per: int, rank: int, world: int, dtype, device, rest=(), group=None,
                  fill=None):
@@ -68,6 +68,7 @@ class BlockArray:
         self.view = self.buf[:n]
         self.mine = self.buf[rank * per:(rank + 1) * per] if world > 1 else self.view
         self._host = None
+        self._send = None
 
     def data_ptr(self) -> int:
         return self.view.data_ptr()
@@ -91,8 +92,12 @@ class BlockArray:
             dist.all_gather_into_tensor(hb, hm, group=self.group)
             self.buf.copy_(hb, non_blocking=False)
         else:
-            # in place: the input is this rank's block of the output buffer
-            dist.all_gather_into_tensor(self.buf, self.mine, group=self.group)
+            # the owned block goes through a persistent send buffer (a D2D copy
+            # of 1/world of the array) rather than aliasing the output
+            if self._send is None:
+                self._send = torch.empty_like(self.mine)
+            self._send.copy_(self.mine)
+            dist.all_gather_into_tensor(self.buf, self._send, group=self.group)
 
 
 def allreduce_(t: torch.Tensor, world: int, group=None, stream=None):

@@ -251,6 +251,9 @@ def _gen_once(env, v, W, s0, steps, warmup):
     return ms, st
 
 
+GEN_HEAP_FULL = False  # --gen-heap-full: the device-heap arm also at 4096^2 (~6 min of device `new`)
+
+
 def app_gen(env, variants, pk, cpu=True, steps=20, warmup=3, small=False):
     W = 256 if small else 4096
     s0 = synth.soup(W, W, seed=42)
@@ -258,7 +261,7 @@ def app_gen(env, variants, pk, cpu=True, steps=20, warmup=3, small=False):
                      f"{env.world} GPU(s) + halo rows; 3 x 16.8M objects (> L2)",
            "calls_per_step": W * W, "variants": {}}
     states = {}
-    for v in _variants(env, variants, heap_ok=False):
+    for v in _variants(env, variants, heap_ok=GEN_HEAP_FULL or small):
         ms, states[v] = _gen_once(env, v, W, s0, steps, warmup)
         row["variants"][v] = {"ms_per_step": ms, "calls_per_s": W * W / (ms / 1e3)}
     ref = next(iter(states.values()))
@@ -267,7 +270,7 @@ def app_gen(env, variants, pk, cpu=True, steps=20, warmup=3, small=False):
     if base:
         row["speedup_vs_cuda_packed"] = {k: base / x["ms_per_step"] for k, x in row["variants"].items()}
     # same-config comparison with the device-heap arm (3 x 4.2M `new`s fit the bench budget)
-    if "cuda" in variants and env.world == 1:
+    if "cuda" in variants and env.world == 1 and not GEN_HEAP_FULL:
         W2 = 128 if small else 2048
         s2 = synth.soup(W2, W2, seed=42)
         sub = {"config": f"{W2}x{W2} (all five variants incl. the device-heap CUDA arm; the heap arm at "
@@ -455,7 +458,11 @@ if __name__ == "__main__":
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--out", default=None)
     ap.add_argument("--small", action="store_true", help="code-path test sizes")
+    ap.add_argument("--gen-heap-full", action="store_true",
+                    help="GEN: the device-heap CUDA arm at 4096^2 too (3 x 16.8M device `new`s, ~6 min)")
     a = ap.parse_args()
+    global GEN_HEAP_FULL
+    GEN_HEAP_FULL = a.gen_heap_full
     from paper_conf_asplos_zhangar21_b200 import vf
     ctx = vf.Ctx(0, cuda_heap_bytes=16 << 30)
     env = Env(ctx)

@@ -112,7 +112,7 @@ def main():
           "stall long-sb | stall barrier |",
           "|" + "---|" * 18]
     for rep in a.reports:
-        variant = os.path.basename(rep).split("_")[1]
+        variant = os.path.basename(rep).split("_")[1]  # prof_<variant>_T4[.ncu-rep|.raw.csv]
         for d in raw(rep):
             n = a.n
             traffic = d.get("dram_read", 0) + d.get("dram_write", 0)
