@@ -706,7 +706,8 @@ vf_status vf_checksum_i32(const int32_t* vals_dev, uint64_t n, long long* out_de
 /* Benchmark / ablation knobs of the COAL / TYPEPTR kernels (process-wide):
  * "unroll" = objects per thread (1, 2, 4; -1 = app default); "prefetch" =
  * object-line warm-up before the type groups (0 none, 1 prefetch.global.L1,
- * 2 L1-allocating load; -1 = app default); "regroup" = 1 (default) sorts
+ * 2 L1-allocating load, 3 = 2 issued one tile ahead with the pointers two
+ * tiles ahead (sorted kernel); -1 = app default); "regroup" = 1 (default) sorts
  * each CTA tile by type in shared memory before the calls, 0 groups within
  * warps only; "pipeline" = 1 streams the pointer array through a TMA /
  * mbarrier ring in shared memory (regroup 0 only), 0 (default) uses plain

@@ -483,44 +483,70 @@ __global__ void __launch_bounds__(kBlock, MinBlocks<App>::value) k_dispatch_sort
 
   // Light methods keep the NEXT tile's pointers in flight (registers) while
   // this tile is resolved, sorted and called: the pointer stream never waits
-  // for the tile's barriers.
+  // for the tile's barriers. PF = 3 (deep): pointers TWO tiles ahead and the
+  // next tile already resolved with its object lines warmed (L1-allocating
+  // loads) before this tile's sort and calls, so one tile of object traffic is
+  // always in flight behind the current tile's work.
   constexpr bool kAhead = ((HeavyMaskOf<App>::value >> M) & 1u) == 0;
+  constexpr bool kDeep = kAhead && PF == 3;
   const uint64_t stride = (uint64_t)gridDim.x * TILE;
-  uint64_t pn[U];
-  if constexpr (kAhead) {
+  auto load_ptrs = [&](uint64_t b, uint64_t (&q)[U]) {
 #pragma unroll
     for (int j = 0; j < U; ++j) {
-      const uint64_t idx = (uint64_t)blockIdx.x * TILE + (uint64_t)j * kBlock + threadIdx.x;
-      pn[j] = idx < n ? ldg_u64(objs + idx) : 0ull;
+      const uint64_t idx = b + (uint64_t)j * kBlock + threadIdx.x;
+      q[j] = idx < n ? ldg_u64(objs + idx) : 0ull;
     }
+  };
+  // pointers -> (type, address) incl. the vTable* fallback; warm the object lines
+  auto resolve_warm = [&](const uint64_t (&q)[U], uint64_t (&aa)[U], uint32_t (&tt)[U], uint32_t (&ww)[U]) {
+#pragma unroll
+    for (int j = 0; j < U; ++j) {
+      tt[j] = q[j] ? R::resolve(smem, tbl, q[j], aa[j], hint) : kNF;
+      if (!q[j]) aa[j] = 0;
+      const bool fb = tt[j] >= (uint32_t)App::kTypes && q[j] != 0;
+      if (__any_sync(0xffffffffu, fb)) {
+        if (fb) tt[j] = type_from_vptr<App>(aa[j], tbl);
+      }
+      ww[j] = 0;
+      if constexpr (PF >= 2) {
+        if (tt[j] < (uint32_t)App::kTypes) ww[j] = *reinterpret_cast<const uint32_t*>(aa[j] + 8);
+      }
+    }
+  };
+  uint64_t pn[U];
+  uint64_t an[U];
+  uint32_t tn[U], wn[U];
+  if constexpr (kDeep) {
+    uint64_t p0[U];
+    load_ptrs((uint64_t)blockIdx.x * TILE, p0);
+    load_ptrs((uint64_t)blockIdx.x * TILE + stride, pn);
+    resolve_warm(p0, an, tn, wn);
+  } else if constexpr (kAhead) {
+    load_ptrs((uint64_t)blockIdx.x * TILE, pn);
   }
   for (uint64_t base = (uint64_t)blockIdx.x * TILE; base < n; base += stride) {
     // A: pointers -> (type, address); warm the object lines
     uint64_t p[U], a[U];
     uint32_t t[U], w[U], rank[U];
+    if constexpr (kDeep) {
 #pragma unroll
-    for (int j = 0; j < U; ++j) {
+      for (int j = 0; j < U; ++j) {
+        a[j] = an[j];
+        t[j] = tn[j];
+        w[j] = wn[j];
+        p[j] = pn[j];  // tile k+1
+      }
+      load_ptrs(base + 2 * stride, pn);  // tile k+2
+      resolve_warm(p, an, tn, wn);       // tile k+1: resolved, lines in flight
+    } else {
       if constexpr (kAhead) {
-        p[j] = pn[j];
-        const uint64_t idx = base + stride + (uint64_t)j * kBlock + threadIdx.x;
-        pn[j] = idx < n ? ldg_u64(objs + idx) : 0ull;
-      } else {
-        const uint64_t idx = base + (uint64_t)j * kBlock + threadIdx.x;
-        p[j] = idx < n ? ldg_u64(objs + idx) : 0ull;
-      }
-    }
 #pragma unroll
-    for (int j = 0; j < U; ++j) {
-      t[j] = p[j] ? R::resolve(smem, tbl, p[j], a[j], hint) : kNF;
-      if (!p[j]) a[j] = 0;
-      const bool fb = t[j] >= (uint32_t)App::kTypes && p[j] != 0;
-      if (__any_sync(0xffffffffu, fb)) {
-        if (fb) t[j] = type_from_vptr<App>(a[j], tbl);
+        for (int j = 0; j < U; ++j) p[j] = pn[j];
+        load_ptrs(base + stride, pn);
+      } else {
+        load_ptrs(base, p);
       }
-      w[j] = 0;
-      if constexpr (PF == 2) {
-        if (t[j] < (uint32_t)App::kTypes) w[j] = *reinterpret_cast<const uint32_t*>(a[j] + 8);
-      }
+      resolve_warm(p, a, t, w);
     }
     // Tiles whose warps are already type-uniform (sorted input, run interiors)
     // skip the sort: one barrier instead of four. Both cases reach the SAME
@@ -948,11 +974,13 @@ cudaError_t launch_grouped_pf(int pf, const uint64_t* objs, uint64_t n, const Ar
                               const DevTable& tbl, cudaStream_t s) {
   if constexpr (App::kTypes > 1) {
     if (tuning().regroup != 0) {
+      if (pf == 3) return launch_sorted<App, M, R, U, 3>(objs, n, args, tbl, s);
       if (pf == 2) return launch_sorted<App, M, R, U, 2>(objs, n, args, tbl, s);
       return launch_sorted<App, M, R, U, 0>(objs, n, args, tbl, s);
     }
   }
   // TMA needs a 16-byte aligned source; the pipeline is the default when it applies
+  if (pf == 3) pf = 2;  // the deep pipeline is the sorted kernel's
   if (tuning().pipeline != 0 && (reinterpret_cast<uintptr_t>(objs) & 15) == 0) {
     if (pf == 0) return launch_pipe<App, M, R, U, 0, 4>(objs, n, args, tbl, s);
     if (pf == 1) return launch_pipe<App, M, R, U, 1, 4>(objs, n, args, tbl, s);

@@ -42,7 +42,7 @@ def test_micro_parity(ctx, variant, T, order):
 
 
 @pytest.mark.parametrize("unroll", [1, 2, 4])
-@pytest.mark.parametrize("prefetch", [0, 1, 2])
+@pytest.mark.parametrize("prefetch", [0, 1, 2, 3])
 @pytest.mark.parametrize("pipeline,regroup", [(0, 0), (1, 0), (0, 1)])
 @pytest.mark.parametrize("variant", ["coal", "typeptr"])
 @pytest.mark.parametrize("n", [50_000 + 3, 1024 * 300, 100])
@@ -274,3 +274,26 @@ def test_dispatch_host_matches_closed_form(variant, chunk):
     assert np.array_equal(got, init + R * (types.astype(np.int32) + 1))
     assert torch.equal(staging, m.objs)
     c.close()
+
+
+@pytest.mark.parametrize("unroll", [1, 2, 4])
+@pytest.mark.parametrize("variant,T", [("coal", 4), ("typeptr", 4), ("coal", 32), ("typeptr", 32)])
+def test_micro_deep_pipeline_many_waves(ctx, unroll, variant, T):
+    """prefetch 3 (pointers two tiles ahead, the next tile resolved and warmed
+    during this one): inputs spanning >= 3 persistent-grid waves so every CTA
+    runs the steady state, the last two tiles and a ragged tail."""
+    n = 3 * 148 * 8 * 1024 + 77
+    R = 2
+    types = synth.micro_types(n, T, "random", seed=5)
+    init = synth.micro_init(n, seed=5)
+    vf.set_tuning("unroll", unroll)
+    vf.set_tuning("prefetch", 3)
+    try:
+        m = apps.Micro(ctx, n, T, variant=variant, types_np=types, init_np=init)
+        for _ in range(R):
+            m.step()
+        got = m.values().cpu().numpy()
+        assert np.array_equal(got, init + R * (types.astype(np.int32) + 1))  # closed form (W0)
+    finally:
+        vf.set_tuning("unroll", -1)
+        vf.set_tuning("prefetch", -1)

@@ -36,6 +36,9 @@ def main():
     ap.add_argument("--n", type=int, default=1 << 26)
     ap.add_argument("--Ts", default="4,32")
     ap.add_argument("--out", default="gpurun_out/sweep_knobs")
+    ap.add_argument("--regroups", default="1,0")
+    ap.add_argument("--unrolls", default="1,2,4")
+    ap.add_argument("--pfs", default="0,1,2", help="prefetch values (3 = deep pipeline, sorted kernel)")
     a = ap.parse_args()
     ctx = vf.Ctx(0, cuda_heap_bytes=1 << 30)
     rows = []
@@ -44,9 +47,9 @@ def main():
         init = synth.micro_init(a.n, seed=42)
         for v in ("coal", "typeptr"):
             m = apps.Micro(ctx, a.n, T, variant=v, types_np=types, init_np=init)
-            for rg in (1, 0):
-                for u in (1, 2, 4):
-                    for pf in (0, 1, 2):
+            for rg in [int(x) for x in a.regroups.split(",")]:
+                for u in [int(x) for x in a.unrolls.split(",")]:
+                    for pf in [int(x) for x in a.pfs.split(",")]:
                         vf.set_tuning("regroup", rg)
                         vf.set_tuning("unroll", u)
                         vf.set_tuning("prefetch", pf)
