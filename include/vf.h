@@ -721,7 +721,7 @@ vf_status vf_checksum_i32(const int32_t* vals_dev, uint64_t n, long long* out_de
  * grids of <= 2^17 cells in ONE thread-block cluster (state in distributed
  * shared memory, hardware cluster barrier), 0 (default; measured faster on
  * B200: a 16-SM cluster serialises 4 cells per thread) always uses the
- * cooperative grid-barrier kernel; "ray_rays" = 2 (default) or 4: pixels
+ * cooperative grid-barrier kernel; "ray_rays" = 4 (default) or 2: pixels
  * (rays) per thread in both ray-tracer kernels.
  * The unroll / prefetch / pipeline knobs apply to config 2's app (micro);
  * the other apps run their default launch configuration.

@@ -122,7 +122,7 @@ struct Tuning {
   int call = 0;       // COAL / TypePointer: 0 grouped direct call, 1 indirect CALL via vFunc* table
   int persistent = -1; // grouped kernels: 1 persistent grid, 0 one tile per CTA, -1 app default (kHeavyMask)
   int cluster = 0;     // vf_gol_run: 1 one thread-block cluster (state in DSMEM) when the grid fits
-  int ray_rays = 2;       // ray kernels: pixels (rays) per thread, 2 or 4
+  int ray_rays = 4;       // ray kernels: pixels (rays) per thread, 2 or 4
 };
 Tuning& tuning();
 

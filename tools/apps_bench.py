@@ -461,8 +461,7 @@ if __name__ == "__main__":
     ap.add_argument("--gen-heap-full", action="store_true",
                     help="GEN: the device-heap CUDA arm at 4096^2 too (3 x 16.8M device `new`s, ~6 min)")
     a = ap.parse_args()
-    global GEN_HEAP_FULL
-    GEN_HEAP_FULL = a.gen_heap_full
+    globals()["GEN_HEAP_FULL"] = a.gen_heap_full
     from paper_conf_asplos_zhangar21_b200 import vf
     ctx = vf.Ctx(0, cuda_heap_bytes=16 << 30)
     env = Env(ctx)
