@@ -680,6 +680,26 @@ typedef struct {
 } vf_collide_grid_args;
 uint64_t vf_collide_tmp_words(uint32_t N, uint32_t G);
 vf_status vf_collide_grid(const vf_collide_grid_args* args, void* stream);
+/* Multi-GPU exchange after update. merge() of body i reads near,
+ * Pm, Vm of j = near[i] only when near[j] >= 0, so a rank owning bodies
+ * [lo, hi) packs just those with near >= 0 (vf_collide_pack_near: appends
+ * entries to out_dev at *count_dev, order unspecified), the packed lists are
+ * all-gathered (rank r's segment of `seg` entries holds counts_dev[r] valid
+ * ones), and vf_collide_unpack_near resets near[] of every body outside
+ * [lo, hi) to -1 and then writes the received entries (own ones skipped). */
+typedef struct {
+  uint32_t id;
+  int32_t near;
+  uint32_t pad[2];
+  float Pm[4]; /* post-update position + mass */
+  float Vm[4]; /* post-update velocity        */
+} vf_collide_near_entry;
+vf_status vf_collide_pack_near(uint32_t lo, uint32_t hi, const int32_t* near_dev, const float* Pm_dev,
+                               const float* Vm_dev, vf_collide_near_entry* out_dev, uint32_t* count_dev,
+                               void* stream);
+vf_status vf_collide_unpack_near(const vf_collide_near_entry* in_dev, uint32_t nseg, uint32_t seg,
+                                 const int64_t* counts_dev, uint32_t N, uint32_t lo, uint32_t hi,
+                                 int32_t* near_dev, float* Pm_dev, float* Vm_dev, void* stream);
 
 /* Graph helpers: BFS start state (depth = -1 except depth[src] = 0, queue =
  * src's nch work entries (vobj[src], chunks 0..nch-1), *count = nch), iota

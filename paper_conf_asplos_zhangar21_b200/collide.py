@@ -9,8 +9,9 @@ positions + masses are float4 arrays indexed by body id. One step:
 
 Multi-GPU (§8e): bodies are split into contiguous id blocks. Every rank holds
 all positions and builds the (replicated) grid; it dispatches its own bodies
-only. After update the owned slices of Pm / Vm / near are all-gathered (a
-merge partner may live on another rank); after merge the owned slices of P.
+only. After update only the bodies with a merge candidate (near >= 0, a few
+per mille) travel, as packed (id, near, Pm, Vm) entries (a merge partner may
+live on another rank); after merge the owned slices of P are all-gathered.
 """
 from __future__ import annotations
 
@@ -49,6 +50,7 @@ class Collide:
         self._Vm = xc.BlockArray(dtype=torch.float32, rest=(4,), fill=0.0, **blk)
         self._near = xc.BlockArray(dtype=torch.int32, fill=-1, **blk)
         self.P, self.Pm, self.Vm, self.near = self._P.view, self._Pm.view, self._Vm.view, self._near.view
+        self._vg = None  # variable-length exchange after update (created on first use)
         self.Ps = torch.zeros((max(N, 1), 4), **f4)
         ncell = self.G ** 3
         u32 = dict(dtype=torch.int32, device=dev)
@@ -94,9 +96,30 @@ class Collide:
                                               self.n_owned, self._upd, vf._stream(stream)), "collide update")
 
     def exchange_update(self, stream=None):
-        if self.world > 1 and self.exchange:
-            for b in (self._Pm, self._Vm, self._near):
-                b.gather(stream)
+        """merge() of body i reads near / Pm / Vm of j = near[i] only when j has a
+        candidate too (near[j] >= 0): only those bodies' entries travel
+        (vf_collide_pack_near -> all-gather of the packed lists ->
+        vf_collide_unpack_near), a few per mille of the bodies instead of the
+        whole 36 B/body arrays."""
+        if not (self.world > 1 and self.exchange):
+            return
+        L = vf.lib()
+        s = vf._stream(stream)
+        if self._vg is None:
+            self._vg = xc.VarGather(self.world, ctypes.sizeof(vf.collide_near_entry), self.dev, self.group)
+            self._cnt = torch.zeros(1, dtype=torch.int32, device=self.dev)
+        send = self._vg.send_buffer(max(self.per, 1))  # worst case: every owned body has a candidate
+        with xc._on(stream, self._cnt):
+            self._cnt.zero_()
+        self.ctx._check(L.vf_collide_pack_near(self.lo, self.hi, self.near.data_ptr(), self.Pm.data_ptr(),
+                                               self.Vm.data_ptr(), send.data_ptr(), self._cnt.data_ptr(), s),
+                        "collide pack")
+        with xc._on(stream, self._cnt):
+            count = int(self._cnt.item())
+        recv, counts, seg = self._vg.gather(count, stream)
+        self.ctx._check(L.vf_collide_unpack_near(recv.data_ptr(), self.world, seg, counts.data_ptr(), self.N,
+                                                 self.lo, self.hi, self.near.data_ptr(), self.Pm.data_ptr(),
+                                                 self.Vm.data_ptr(), s), "collide unpack")
 
     def merge(self, stream=None):
         """Step (2): one virtual merge() per owned active body."""

@@ -424,6 +424,90 @@ static cudaError_t scan_u32(const uint32_t* in, uint32_t* out, uint64_t n, uint3
 
 }  // namespace vf
 
+namespace vf {
+namespace collide {
+// Multi-GPU exchange after update: merge() on body i reads
+// near[j], Pm[j], Vm[j] of its nearest body j = near[i] only when j has a
+// partner (near[j] >= 0), so only those bodies' entries travel.
+__global__ void k_pack_near(uint32_t lo, uint32_t hi, const int32_t* __restrict__ near, const float4* __restrict__ Pm,
+                            const float4* __restrict__ Vm, vf_collide_near_entry* __restrict__ out,
+                            uint32_t* __restrict__ count) {
+  const uint32_t lane = threadIdx.x & 31u;
+  for (uint64_t b = lo + (uint64_t)blockIdx.x * blockDim.x; b < hi; b += (uint64_t)gridDim.x * blockDim.x) {
+    const uint64_t i = b + threadIdx.x;
+    const bool take = i < hi && near[i] >= 0;
+    const uint32_t m = __ballot_sync(0xffffffffu, take);
+    if (!m) continue;
+    const uint32_t leader = __ffs(m) - 1;
+    uint32_t base = 0;
+    if (lane == leader) base = atomicAdd(count, (uint32_t)__popc(m));
+    base = __shfl_sync(0xffffffffu, base, leader);
+    if (take) {
+      vf_collide_near_entry e;
+      e.id = (uint32_t)i;
+      e.near = near[i];
+      e.pad[0] = e.pad[1] = 0;
+      const float4 pm = Pm[i], vm = Vm[i];
+      e.Pm[0] = pm.x; e.Pm[1] = pm.y; e.Pm[2] = pm.z; e.Pm[3] = pm.w;
+      e.Vm[0] = vm.x; e.Vm[1] = vm.y; e.Vm[2] = vm.z; e.Vm[3] = vm.w;
+      out[base + __popc(m & ((1u << lane) - 1u))] = e;
+    }
+  }
+}
+// near[] of every body outside [lo, hi) back to -1 (no partner) ...
+__global__ void k_reset_near(uint32_t N, uint32_t lo, uint32_t hi, int32_t* __restrict__ near) {
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < N; i += (uint64_t)gridDim.x * blockDim.x)
+    if (i < lo || i >= hi) near[i] = -1;
+}
+// ... then the received entries: slot k of rank r's segment is valid iff k < counts[r]
+__global__ void k_unpack_near(const vf_collide_near_entry* __restrict__ in, uint32_t nseg, uint32_t seg,
+                              const int64_t* __restrict__ counts, uint32_t lo, uint32_t hi, int32_t* __restrict__ near,
+                              float4* __restrict__ Pm, float4* __restrict__ Vm) {
+  for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < (uint64_t)nseg * seg;
+       k += (uint64_t)gridDim.x * blockDim.x) {
+    if ((int64_t)(k % seg) >= counts[k / seg]) continue;
+    const vf_collide_near_entry e = in[k];
+    if (e.id >= lo && e.id < hi) continue;  // own entries are already in place
+    near[e.id] = e.near;
+    Pm[e.id] = make_float4(e.Pm[0], e.Pm[1], e.Pm[2], e.Pm[3]);
+    Vm[e.id] = make_float4(e.Vm[0], e.Vm[1], e.Vm[2], e.Vm[3]);
+  }
+}
+}  // namespace collide
+}  // namespace vf
+
+extern "C" vf_status vf_collide_pack_near(uint32_t lo, uint32_t hi, const int32_t* near_dev, const float* Pm_dev,
+                                          const float* Vm_dev, vf_collide_near_entry* out_dev, uint32_t* count_dev,
+                                          void* stream) {
+  if (hi < lo || (hi > lo && (!near_dev || !Pm_dev || !Vm_dev || !out_dev || !count_dev))) return VF_ERR_INVALID;
+  if (hi == lo) return VF_OK;
+  vf::collide::k_pack_near<<<(unsigned)vf::num_sms() * 4, 256, 0, (cudaStream_t)stream>>>(
+      lo, hi, near_dev, reinterpret_cast<const float4*>(Pm_dev), reinterpret_cast<const float4*>(Vm_dev), out_dev,
+      count_dev);
+  vf::note_launch();
+  return cudaGetLastError() == cudaSuccess ? VF_OK : VF_ERR_CUDA;
+}
+
+extern "C" vf_status vf_collide_unpack_near(const vf_collide_near_entry* in_dev, uint32_t nseg, uint32_t seg,
+                                            const int64_t* counts_dev, uint32_t N, uint32_t lo, uint32_t hi,
+                                            int32_t* near_dev, float* Pm_dev, float* Vm_dev, void* stream) {
+  if (!near_dev || !Pm_dev || !Vm_dev || (nseg && seg && (!in_dev || !counts_dev)) || hi < lo || hi > N)
+    return VF_ERR_INVALID;
+  const cudaStream_t s = (cudaStream_t)stream;
+  const unsigned grid = (unsigned)vf::num_sms() * 4;
+  if (N) {
+    vf::collide::k_reset_near<<<grid, 256, 0, s>>>(N, lo, hi, near_dev);
+    vf::note_launch();
+  }
+  if (nseg && seg) {
+    vf::collide::k_unpack_near<<<grid, 256, 0, s>>>(in_dev, nseg, seg, counts_dev, lo, hi, near_dev,
+                                                     reinterpret_cast<float4*>(Pm_dev),
+                                                     reinterpret_cast<float4*>(Vm_dev));
+    vf::note_launch();
+  }
+  return cudaGetLastError() == cudaSuccess ? VF_OK : VF_ERR_CUDA;
+}
+
 extern "C" uint64_t vf_collide_tmp_words(uint32_t N, uint32_t G) {
   const uint64_t ncell = (uint64_t)G * G * G;
   const uint64_t big = ncell > N ? ncell : N;

@@ -387,7 +387,7 @@ DevTable dev_table(vf_ctx* c, uint32_t app) {
   for (uint32_t j = 0; j < kTableInline; ++j) {
     const bool v = j < t.K && t.K <= kTableInline;
     d.in_start[j] = v ? t.rows[j].start : ~0ull;
-    d.in_end[j] = v ? t.rows[j].end : 0ull;
+    d.in_len[j] = v ? t.rows[j].end - t.rows[j].start : 0ull;
     d.in_type[j] = v ? t.rows[j].type_id : VF_NOT_FOUND;
   }
   return d;

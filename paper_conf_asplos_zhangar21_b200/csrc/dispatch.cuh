@@ -127,11 +127,13 @@ struct ResolveCOAL {
     p = a;
     (void)hint;
     if (tbl.K <= kTableInline) {
+      // p in [start, end) <=> (p - start) < (end - start), unsigned: one
+      // 64-bit subtract and one 64-bit compare per row
       uint32_t t = kNF;
 #pragma unroll
       for (uint32_t j = 0; j < kTableInline; ++j) {
         if (j >= tbl.K) break;  // uniform
-        t = (p >= tbl.in_start[j] && p < tbl.in_end[j]) ? tbl.in_type[j] : t;
+        t = (p - tbl.in_start[j] < tbl.in_len[j]) ? tbl.in_type[j] : t;
       }
       return t;
     }

@@ -35,7 +35,7 @@ struct DevTable {
   uint32_t ntypes;
   uint32_t active_types;  // concrete types with live objects (launch heuristics)
   uint64_t in_start[kTableInline];  // rows 0..K-1 when K <= kTableInline
-  uint64_t in_end[kTableInline];
+  uint64_t in_len[kTableInline];    // end - start (0 for padding rows)
   uint32_t in_type[kTableInline];
 };
 

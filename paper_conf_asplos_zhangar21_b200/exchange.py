@@ -14,6 +14,8 @@ exchanged here, with NO per-call allocation:
   positions all use it.
 * ``HaloRows``: the GEN row slabs' halo exchange, ``batch_isend_irecv`` of
   one boundary row to each neighbour slab per generation.
+* ``VarGather``: variable-length row lists (collision: only the bodies with a
+  merge candidate travel after update).
 * ``allreduce_``: in-place sum (BFS "changed", PR dangling mass).
 
 CPU tests drive the same code over ``gloo`` process groups. gloo cannot move
@@ -98,6 +100,54 @@ class BlockArray:
                 self._send = torch.empty_like(self.mine)
             self._send.copy_(self.mine)
             dist.all_gather_into_tensor(self.buf, self._send, group=self.group)
+
+
+class VarGather:
+    """All-gather of variable-length row lists (persistent, grown on demand):
+    every rank contributes `count` rows; the result holds world segments of
+    max(count) rows each, rank r's first counts[r] rows valid. Two collectives
+    (the counts, then the padded rows) and one host read of the counts."""
+
+    def __init__(self, world: int, row_bytes: int, device, group=None):
+        self.world, self.row_bytes, self.device, self.group = world, row_bytes, device, group
+        self.counts = torch.zeros(world, dtype=torch.int64, device=device)
+        self._send = self._recv = None
+        self._host = None
+
+    def send_buffer(self, rows: int) -> torch.Tensor:
+        """A (rows x row_bytes) uint8 buffer to pack into (kept across calls)."""
+        if self._send is None or self._send.shape[0] < rows:
+            grown = torch.empty((max(rows, 1), self.row_bytes), dtype=torch.uint8, device=self.device)
+            if self._send is not None:
+                grown[:self._send.shape[0]].copy_(self._send)  # keep what was packed
+            self._send = grown
+        return self._send
+
+    def gather(self, count: int, stream=None):
+        """-> (recv uint8[world * seg, row_bytes], counts int64[world] on the device, seg)."""
+        dist = _dist()
+        with _on(stream, self.counts):
+            mine = torch.tensor([count], dtype=torch.int64, device=self.device)
+            staged = _staged(self.counts, self.group)
+            if staged:
+                hc = torch.empty(self.world, dtype=torch.int64)
+                dist.all_gather_into_tensor(hc, mine.cpu(), group=self.group)
+                self.counts.copy_(hc)
+            else:
+                dist.all_gather_into_tensor(self.counts, mine, group=self.group)
+                hc = self.counts.cpu()
+            seg = max(int(hc.max()), 1)
+            send = self.send_buffer(seg)[:seg]
+            if self._recv is None or self._recv.shape[0] < self.world * seg:
+                self._recv = torch.empty((self.world * seg, self.row_bytes), dtype=torch.uint8, device=self.device)
+            recv = self._recv[:self.world * seg]
+            if staged:
+                hr = torch.empty(recv.shape, dtype=torch.uint8)
+                dist.all_gather_into_tensor(hr, send.cpu(), group=self.group)
+                recv.copy_(hr)
+            else:
+                dist.all_gather_into_tensor(recv, send, group=self.group)
+        return recv, self.counts, seg
 
 
 def allreduce_(t: torch.Tensor, world: int, group=None, stream=None):

@@ -43,6 +43,7 @@ SYMBOLS = [
     "vf_gol_neighbors", "vf_gol_swap", "vf_gen_swap", "vf_checksum_i32", "vf_launch_count", "vf_set_tuning",
     "vf_graph_bfs_init", "vf_iota_u32", "vf_fill_f32", "vf_ray_render", "vf_gol_step", "vf_gen_step", "vf_gen_step_rows", "vf_gol_run", "vf_dispatch_host",
     "vf_dispatch_concord", "vf_micro_branch", "vf_collide_tmp_words", "vf_collide_grid",
+    "vf_collide_pack_near", "vf_collide_unpack_near",
 ]
 APP_RAY = 4
 APP_TRAF = 5
@@ -109,6 +110,11 @@ class collide_grid_args(ctypes.Structure):
                 ("cell_start_dev", ctypes.c_void_p), ("list_dev", ctypes.c_void_p), ("Ps_dev", ctypes.c_void_p),
                 ("slot_dev", ctypes.c_void_p), ("tmp_dev", ctypes.c_void_p), ("objs_dev", ctypes.c_void_p), ("id_lo", ctypes.c_uint32),
                 ("id_hi", ctypes.c_uint32), ("order_dev", ctypes.c_void_p), ("active_dev", ctypes.c_void_p)]
+
+
+class collide_near_entry(ctypes.Structure):
+    _fields_ = [("id", ctypes.c_uint32), ("near", ctypes.c_int32), ("pad", ctypes.c_uint32 * 2),
+                ("Pm", ctypes.c_float * 4), ("Vm", ctypes.c_float * 4)]
 
 
 class traf_cell_args(ctypes.Structure):
@@ -287,6 +293,8 @@ def lib(required: bool = True):
         "vf_collide_grid": (I, [ctypes.POINTER(collide_grid_args), P]),
         "vf_gen_step": (I, [P, I, U32, U32, I, P, P, P, P, P, P, P, U32, U32, U32, P]),
         "vf_gen_step_rows": (I, [P, I, U32, U32, I, U32, U32, P, P, P, P, P, P, P, U32, U32, U32, P]),
+        "vf_collide_pack_near": (I, [U32, U32, P, P, P, P, P, P]),
+        "vf_collide_unpack_near": (I, [P, U32, U32, P, U32, U32, U32, P, P, P, P]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)

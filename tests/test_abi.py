@@ -105,7 +105,7 @@ def test_arg_struct_layouts_match_header(tmp_path):
                "vf_graph_en_pr_args": vf.graph_en_pr_args, "vf_edge_args": vf.edge_args,
                "vf_edge_resolver": vf.edge_resolver, "vf_graph_bfs_args": vf.graph_bfs_args,
                "vf_graph_cc_args": vf.graph_cc_args, "vf_graph_pr_args": vf.graph_pr_args,
-               "vf_graph_bfs_bits_args": vf.graph_bfs_bits_args}
+               "vf_graph_bfs_bits_args": vf.graph_bfs_bits_args, "vf_collide_near_entry": vf.collide_near_entry}
     lines = ['#include <stdio.h>', '#include <stddef.h>', f'#include "{HDR}"', "int main(void) {"]
     for cname, py in structs.items():
         lines.append(f'  printf("{cname} %zu\\n", sizeof({cname}));')

@@ -221,3 +221,41 @@ def test_exchange_blockarray_halo_gloo(world):
                     assert (st[row % H] == row % H).all(), (torus, row)
             untouched = [q for q in range(H) if not (r0 - 1 <= q <= r1) and not (torus and q in ((r0 - 1) % H, r1 % H))]
             assert all((st[q] == 255).all() for q in untouched)
+
+
+def _vargather_worker(rank, world, port, outdir):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    from paper_conf_asplos_zhangar21_b200 import exchange
+    vg = exchange.VarGather(world, 6, "cpu")
+    out = {}
+    for step, extra in enumerate((0, 3, 1)):  # the send buffer grows and keeps its content
+        count = rank * 2 + extra
+        send = vg.send_buffer(count)
+        send[:count] = torch.arange(count * 6, dtype=torch.uint8).view(count, 6) + 10 * rank
+        recv, counts, seg = vg.gather(count)
+        out[f"recv{step}"] = recv.numpy().copy()
+        out[f"counts{step}"] = counts.numpy().copy()
+        out[f"seg{step}"] = np.array([seg])
+    np.savez(os.path.join(outdir, f"v{rank}.npz"), **out)
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_exchange_vargather_gloo(world):
+    """exchange.VarGather (collision's post-update exchange): variable-length
+    row lists, every rank's rows in its own segment, counts all-gathered."""
+    with tempfile.TemporaryDirectory() as td:
+        mp.spawn(_vargather_worker, args=(world, _free_port(), td), nprocs=world, join=True)
+        res = [dict(np.load(os.path.join(td, f"v{r}.npz"))) for r in range(world)]
+    for step, extra in enumerate((0, 3, 1)):
+        counts = [r * 2 + extra for r in range(world)]
+        for d in res:
+            assert list(d[f"counts{step}"]) == counts
+            seg = int(d[f"seg{step}"][0])
+            assert seg == max(max(counts), 1)
+            recv = d[f"recv{step}"]
+            for r, c in enumerate(counts):
+                want = np.arange(c * 6, dtype=np.uint8).reshape(c, 6) + 10 * r
+                assert np.array_equal(recv[r * seg:r * seg + c], want)
