@@ -124,6 +124,28 @@ def _roof(bound, per_call, calls_per_s, pk):
             "per_call": per_call, "peak_source": pk["hbm_src"]}
 
 
+def _ncu(app_variant):
+    """ncu DRAM bytes of the app's dominant kernel (profiles/ncu_apps_summary.json, committed)."""
+    try:
+        return json.load(open(os.path.join(ROOT, "profiles", "ncu_apps_summary.json")))["captures"].get(app_variant)
+    except Exception:
+        return None
+
+
+def _traffic(row, key, variant, pk, launches_per_step=1):
+    """Real-DRAM roofline of a one-kernel step: the captured launch's DRAM bytes
+    (ncu, cold cache) x launches per step / the measured step time."""
+    cap = _ncu(f"{key}_{variant}")
+    ms = row["variants"].get(variant, {}).get("ms_per_step")
+    if not cap or not ms:
+        return
+    b = cap["dram_bytes"] * launches_per_step
+    row["roofline"]["traffic"] = b
+    row["roofline"]["real_dram_gbs"] = b / (ms / 1e3) / 1e9
+    row["roofline"]["real_frac"] = b / (ms / 1e3) / 1e9 / pk["hbm_gbs"]
+    row["roofline"]["traffic_source"] = f"{cap['source']} ({cap['kernel'][:60]}), {variant}"
+
+
 def _cpu(calls, sec, sample):
     import oracle  # bench.py's cpu_baseline leg (tests-only code, timed, never on the product path)
     return {"value": calls / sec, "unit": "calls/s", "cores": oracle.max_threads(), "kind": "oracle",
@@ -281,6 +303,8 @@ def app_gen(env, variants, pk, cpu=True, steps=20, warmup=3, small=False):
         row["same_config_with_heap_cuda"] = _finish(sub)
     best = max(row["variants"].values(), key=lambda x: x["calls_per_s"])["calls_per_s"]
     row["roofline"] = _roof("hbm", 14, best, pk)
+    if not small and env.world == 1:
+        _traffic(row, "gen", "typeptr", pk)  # the fused step is ONE launch per generation
     if cpu and env.rank == 0:
         import oracle
         _, _, _, sec = oracle.gen_run(W, W, s0, 2, threads=oracle.max_threads())
