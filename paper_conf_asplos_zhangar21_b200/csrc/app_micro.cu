@@ -34,7 +34,6 @@ struct App {
   static constexpr int kUnroll = 2;
   static constexpr int kUnrollSorted = 2;
   static constexpr int kPrefetch = 2;
-  static constexpr int kMinBlocks = 6;  // <= 40 registers: 48 resident warps per SM for the sorted tiles
   using Base = MObj;
   template <int K>
   using Type = MObjK<K>;
