@@ -547,9 +547,14 @@ vf_status vf_verify_types(vf_ctx* ctx, uint32_t app, vf_variant v, const uint64_
  * method's argument struct (args_bytes <= VF_MAX_ARGS_BYTES), copied into
  * the kernel parameters. Pointers must be unique for mutating methods.
  * CUDA / SHAREDOA: plain C++ virtual call (vTable* load, vFunc* load,
- * indirect CALL). COAL: range lookup in shared memory. TYPEPTR: tag shift +
- * strip. COAL and TYPEPTR then group the lanes of a warp by type and run
- * each type's body once per warp as a direct, inlined call. */
+ * indirect CALL) on the pointer as given — it must be untagged (a tagged
+ * pointer faults there, as any invalid pointer does in C++). COAL: range
+ * lookup (the kernel-parameter table for K <= 8 rows, else shared memory) of
+ * the pointer's address (a tag, if present, is stripped first). TYPEPTR:
+ * tag shift + strip. COAL and TYPEPTR then group the lanes of a warp by type
+ * and run each type's body once per warp as a direct, inlined call; a
+ * pointer neither rule types (COAL miss, tag 0) falls back to its embedded
+ * vTable*. vf_resolve / vf_verify_types strip tags before any dereference. */
 vf_status vf_dispatch_cuda(vf_ctx* ctx, uint32_t app, uint32_t method, const uint64_t* objs_dev,
                            uint64_t n, const void* args, size_t args_bytes, void* stream);
 vf_status vf_dispatch_sharedoa(vf_ctx* ctx, uint32_t app, uint32_t method,
@@ -728,8 +733,10 @@ vf_status vf_checksum_i32(const int32_t* vals_dev, uint64_t n, long long* out_de
  * object-line warm-up before the type groups (0 none, 1 prefetch.global.L1,
  * 2 L1-allocating load, 3 = 2 issued one tile ahead with the pointers two
  * tiles ahead (sorted kernel); -1 = app default); "regroup" = 1 (default) sorts
- * each CTA tile by type in shared memory before the calls, 0 groups within
- * warps only; "pipeline" = 1 streams the pointer array through a TMA /
+ * each CTA tile by type in shared memory before the calls (4 barriers per
+ * tile), 2 the same sort with 2 barriers per tile (double-buffered histogram
+ * that every warp scans; light methods, prefetch 2), 0 groups within warps
+ * only; "pipeline" = 1 streams the pointer array through a TMA /
  * mbarrier ring in shared memory (regroup 0 only), 0 (default) uses plain
  * per-thread loads; "call" = 1 makes COAL / TYPEPTR CALL the resolved type's
  * vFunc* indirectly (the paper's design, Table 1 row C, Fig. 5b line 4), 0

@@ -443,7 +443,7 @@ vf_status vf_set_tuning(const char* key, int value) {
     if (value < -1 || value > 3) return VF_ERR_INVALID;
     tuning().prefetch = value;
   } else if (!strcmp(key, "regroup")) {
-    if (value < 0 || value > 1) return VF_ERR_INVALID;
+    if (value < 0 || value > 2) return VF_ERR_INVALID;
     tuning().regroup = value;
   } else if (!strcmp(key, "pipeline")) {
     if (value < 0 || value > 1) return VF_ERR_INVALID;

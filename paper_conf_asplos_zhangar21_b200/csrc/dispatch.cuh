@@ -458,14 +458,20 @@ struct SortSmem {
   static constexpr size_t kA = (size_t)kTile * sizeof(uint64_t);   // sorted addresses
   static constexpr size_t kI = (size_t)kTile * sizeof(uint32_t);   // sorted tile-local index
   static constexpr size_t kT = (size_t)kTile * sizeof(uint8_t);    // sorted type
-  static constexpr size_t kH = 68 * sizeof(uint32_t);              // hist[32] + offs[33] (+pad)
+  static constexpr size_t kH = 132 * sizeof(uint32_t);             // hist[32] + offs[33] (+pad) | hist[2][32] (SB 2)
   static size_t bytes(size_t table_bytes) { return align16(table_bytes) + kA + kI + align16(kT) + kH; }
 };
 
-template <class App, int M, class R, int U, int PF>
+// SB = barriers per tile: 4 (rank, scan by one warp, scatter, calls) or, for
+// light methods, 2: the rank atomics go into one of two histograms
+// (alternating per tile) BEFORE the CTA-wide mixed test, whose barrier then
+// also publishes the histogram; every warp scans the 32 counts itself in
+// registers; the other histogram is cleared for the next tile.
+template <class App, int M, class R, int U, int PF, int SB = 4>
 __global__ void __launch_bounds__(kBlock, MinBlocks<App>::value) k_dispatch_sorted(const uint64_t* __restrict__ objs,
                                                             uint64_t n, ArgBlob args, DevTable tbl) {
   static_assert(App::kTypes <= 32, "one warp scans the histogram");
+  static_assert(SB == 4 || (SB == 2 && ((HeavyMaskOf<App>::value >> M) & 1u) == 0), "SB 2: light methods");
   extern __shared__ __align__(16) unsigned char smem[];
   using L = SortSmem<U>;
   constexpr int TILE = L::kTile;
@@ -476,12 +482,13 @@ __global__ void __launch_bounds__(kBlock, MinBlocks<App>::value) k_dispatch_sort
   uint32_t* s_hist = reinterpret_cast<uint32_t*>(smem + tbytes + L::kA + L::kI + align16(L::kT));
   uint32_t* s_offs = s_hist + 32;  // 33 entries: exclusive offsets + total
   if constexpr (R::kNeedsTable) R::stage(smem, tbl);
-  if (threadIdx.x < 32) s_hist[threadIdx.x] = 0;
+  if (threadIdx.x < 64) s_hist[threadIdx.x] = 0;  // (SB 2 uses s_hist[0..63] as two histograms)
   __syncthreads();
   const int lane = threadIdx.x & 31;
   const uint32_t lt_mask = (1u << lane) - 1u;
   uint32_t sink = 0;
   uint32_t hint = 0;  // COAL: last range hit by this lane
+  uint32_t hb = 0;    // SB 2: this tile's histogram
 
   // Light methods keep the NEXT tile's pointers in flight (registers) while
   // this tile is resolved, sorted and called: the pointer stream never waits
@@ -560,6 +567,26 @@ __global__ void __launch_bounds__(kBlock, MinBlocks<App>::value) k_dispatch_sort
       const uint32_t pres = __reduce_or_sync(0xffffffffu, t[j] < (uint32_t)App::kTypes ? (1u << t[j]) : 0u);
       mixed |= (pres & (pres - 1)) != 0;
     }
+    if constexpr (SB == 2) {
+      // the other histogram belongs to the previous tile: its atomics ended
+      // before that tile's first barrier, its reads (C) before its second (or
+      // never, for a type-uniform tile) — clear it for the next tile, whose
+      // atomics start after this tile's first barrier
+      if (threadIdx.x < 32) s_hist[(hb ^ 1u) * 32 + threadIdx.x] = 0;
+      // B (before the CTA-wide test): rank within type into this tile's histogram
+      uint32_t* hist = s_hist + hb * 32;
+#pragma unroll
+      for (int j = 0; j < U; ++j) {
+        const bool ok = t[j] < (uint32_t)App::kTypes;
+        const uint32_t key = ok ? t[j] : 0xFFFFu;
+        const uint32_t peers = __match_any_sync(0xffffffffu, key);
+        const int leader = __ffs(peers) - 1;
+        uint32_t b = 0;
+        if (ok && lane == leader) b = atomicAdd(&hist[t[j]], (uint32_t)__popc(peers));
+        b = __shfl_sync(0xffffffffu, b, leader);
+        rank[j] = b + __popc(peers & lt_mask);
+      }
+    }
     const bool sorted = __syncthreads_or(mixed) != 0;  // CTA-uniform
     if constexpr (((HeavyMaskOf<App>::value >> M) & 1u) == 0) {
       // light bodies: a separate call site for type-uniform tiles (no selects
@@ -570,10 +597,36 @@ __global__ void __launch_bounds__(kBlock, MinBlocks<App>::value) k_dispatch_sort
           sink ^= w[j];
           group_call<App, M>(t[j], a[j], 0ull, base + (uint64_t)j * kBlock + threadIdx.x, args, tbl);
         }
+        hb ^= 1u;
         continue;
       }
     }
-    if (sorted) {
+    uint32_t total2 = 0;
+    if constexpr (SB == 2) {
+      // C: every warp scans the 32 counts in registers; D: scatter
+      const uint32_t h = s_hist[hb * 32 + lane];
+      uint32_t x = h;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= o) x += y;
+      }
+      const uint32_t ex = x - h;
+      total2 = __shfl_sync(0xffffffffu, x, 31);
+#pragma unroll
+      for (int j = 0; j < U; ++j) {
+        const bool ok = t[j] < (uint32_t)App::kTypes;
+        const uint32_t off = __shfl_sync(0xffffffffu, ex, ok ? t[j] : 0u);
+        if (ok) {
+          const uint32_t pos = off + rank[j];
+          s_a[pos] = a[j];
+          s_i[pos] = (uint32_t)(j * kBlock + threadIdx.x);
+          s_t[pos] = (uint8_t)t[j];
+        }
+      }
+      __syncthreads();
+      hb ^= 1u;
+    } else if (sorted) {
       // B: rank within type (warp-aggregated smem atomics)
 #pragma unroll
       for (int j = 0; j < U; ++j) {
@@ -614,7 +667,7 @@ __global__ void __launch_bounds__(kBlock, MinBlocks<App>::value) k_dispatch_sort
       __syncthreads();
     }
     // E: each warp walks 32 consecutive (sorted) entries per j
-    const uint32_t total = sorted ? s_offs[32] : 0u;
+    const uint32_t total = SB == 2 ? total2 : (sorted ? s_offs[32] : 0u);
 #pragma unroll
     for (int j = 0; j < U; ++j) sink ^= w[j];
 #pragma unroll
@@ -636,7 +689,7 @@ __global__ void __launch_bounds__(kBlock, MinBlocks<App>::value) k_dispatch_sort
     }
     // (the next tile's __syncthreads_or orders these reads before its scatter)
   }
-  if constexpr (PF == 2) {
+  if constexpr (PF >= 2) {
     if (sink == 0x8BADF00Du && n == ~0ull) asm volatile("st.global.u32 [%0], %1;" ::"l"(objs), "r"(sink));
   }
 }
@@ -959,10 +1012,10 @@ cudaError_t launch_pipe(const uint64_t* objs, uint64_t n, const ArgBlob& args, c
   return cudaGetLastError();
 }
 
-template <class App, int M, class R, int U, int PF>
+template <class App, int M, class R, int U, int PF, int SB = 4>
 cudaError_t launch_sorted(const uint64_t* objs, uint64_t n, const ArgBlob& args, const DevTable& tbl,
                           cudaStream_t s) {
-  constexpr auto kern = k_dispatch_sorted<App, M, R, U, PF>;
+  constexpr auto kern = k_dispatch_sorted<App, M, R, U, PF, SB>;
   const size_t sm = SortSmem<U>::bytes(R::kNeedsTable ? table_smem(tbl) : 0);
   const int occ = occupancy<kern>(sm);
   const unsigned grid = grid_for(n, (uint64_t)kBlock * U, grid_cap<App, M>(occ));
@@ -976,6 +1029,9 @@ cudaError_t launch_grouped_pf(int pf, const uint64_t* objs, uint64_t n, const Ar
                               const DevTable& tbl, cudaStream_t s) {
   if constexpr (App::kTypes > 1) {
     if (tuning().regroup != 0) {
+      if constexpr (((HeavyMaskOf<App>::value >> M) & 1u) == 0) {
+        if (tuning().regroup == 2 && pf == 2) return launch_sorted<App, M, R, U, 2, 2>(objs, n, args, tbl, s);
+      }
       if (pf == 3) return launch_sorted<App, M, R, U, 3>(objs, n, args, tbl, s);
       if (pf == 2) return launch_sorted<App, M, R, U, 2>(objs, n, args, tbl, s);
       return launch_sorted<App, M, R, U, 0>(objs, n, args, tbl, s);

@@ -43,7 +43,7 @@ def test_micro_parity(ctx, variant, T, order):
 
 @pytest.mark.parametrize("unroll", [1, 2, 4])
 @pytest.mark.parametrize("prefetch", [0, 1, 2, 3])
-@pytest.mark.parametrize("pipeline,regroup", [(0, 0), (1, 0), (0, 1)])
+@pytest.mark.parametrize("pipeline,regroup", [(0, 0), (1, 0), (0, 1), (0, 2)])
 @pytest.mark.parametrize("variant", ["coal", "typeptr"])
 @pytest.mark.parametrize("n", [50_000 + 3, 1024 * 300, 100])
 def test_micro_tuning_knobs(ctx, unroll, prefetch, pipeline, regroup, variant, n):
@@ -297,3 +297,27 @@ def test_micro_deep_pipeline_many_waves(ctx, unroll, variant, T):
     finally:
         vf.set_tuning("unroll", -1)
         vf.set_tuning("prefetch", -1)
+
+
+@pytest.mark.parametrize("unroll", [1, 2, 4])
+@pytest.mark.parametrize("order", ["random", "sorted"])
+@pytest.mark.parametrize("variant,T", [("coal", 4), ("typeptr", 4), ("typeptr", 32)])
+def test_micro_two_barrier_sort_many_waves(ctx, unroll, order, variant, T):
+    """regroup 2 (two barriers per tile: double-buffered histogram, per-warp
+    scans) over >= 3 persistent-grid waves, mixed and type-uniform tiles."""
+    n = 3 * 148 * 8 * 1024 + 77
+    R = 3
+    types = synth.micro_types(n, T, order, seed=6)
+    init = synth.micro_init(n, seed=6)
+    vf.set_tuning("unroll", unroll)
+    vf.set_tuning("prefetch", 2)
+    vf.set_tuning("regroup", 2)
+    try:
+        m = apps.Micro(ctx, n, T, variant=variant, types_np=types, init_np=init)
+        for _ in range(R):
+            m.step()
+        assert np.array_equal(m.values().cpu().numpy(), init + R * (types.astype(np.int32) + 1))
+    finally:
+        vf.set_tuning("unroll", -1)
+        vf.set_tuning("prefetch", -1)
+        vf.set_tuning("regroup", 1)

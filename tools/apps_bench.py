@@ -489,7 +489,8 @@ if __name__ == "__main__":
     from paper_conf_asplos_zhangar21_b200 import vf
     ctx = vf.Ctx(0, cuda_heap_bytes=16 << 30)
     env = Env(ctx)
-    res = run_apps(env, a.apps.split(","), tuple(a.variants.split(",")), cpu=not a.no_cpu,
+    from bench import Clocks  # the same nvidia-smi sampler as the contract line
+    res = run_apps(env, a.apps.split(","), tuple(a.variants.split(",")), cpu=not a.no_cpu, clocks_cls=Clocks,
                    log=lambda n, r: print(json.dumps({n: r}), flush=True), small=a.small)
     if a.out:
         json.dump(res, open(a.out, "w"), indent=1)
