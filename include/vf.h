@@ -749,7 +749,13 @@ vf_status vf_checksum_i32(const int32_t* vals_dev, uint64_t n, long long* out_de
  * shared memory, hardware cluster barrier), 0 (default; measured faster on
  * B200: a 16-SM cluster serialises 4 cells per thread) always uses the
  * cooperative grid-barrier kernel; "ray_rays" = 4 (default) or 2: pixels
- * (rays) per thread in both ray-tracer kernels.
+ * (rays) per thread in both ray-tracer kernels; "gsort" = 1 sorts the whole
+ * dispatch list of a heavy method (long bodies: N-body / collision update,
+ * graph methods) by type before the calls under COAL / TYPEPTR (type from
+ * the pointer; (pointer, index) pairs, index order kept within a type; the
+ * body still receives the entry's original index), 0 sorts per CTA tile
+ * only, -1 (default) = the app's choice (N-body and collision sort the list;
+ * the graph methods, measured no faster, do not).
  * The unroll / prefetch / pipeline knobs apply to config 2's app (micro);
  * the other apps run their default launch configuration.
  * VF_ERR_INVALID for unknown keys / values. */

@@ -141,6 +141,13 @@ cudaError_t rank_hist(const uint32_t* types, uint64_t n, uint32_t ntypes, uint32
   return cudaGetLastError();
 }
 
+cudaError_t scan_type_hist(uint32_t* hist, uint64_t nchunks, uint32_t ntypes, unsigned long long* totals,
+                           cudaStream_t s) {
+  alloc::k_hist_scan<<<1, 32 * 32, 0, s>>>(hist, nchunks, ntypes, totals);
+  note_launch();
+  return cudaGetLastError();
+}
+
 cudaError_t rank_place(const uint32_t* types, uint64_t n, const uint32_t* hist, const PlaceSeg* segs,
                        const uint32_t* seg_first, int tag, uint64_t* out, cudaStream_t s) {
   const uint64_t nb = rank_chunks(n);

@@ -188,6 +188,7 @@ struct App {
   static constexpr int kUnrollSorted = 1;
   static constexpr int kPrefetch = 0;
   static constexpr bool kLean = true;  // default launch configuration only (knob sweeps: micro)
+  static constexpr bool kGridSort = true;  // heavy update: grid-level type sort (measured)
   static constexpr uint32_t kHeavyMask = 1u << VF_COLLIDE_UPDATE;  // one tile per CTA (dispatch.cuh grid_cap)
   static constexpr int kMinBlocks = 5;  // <= 48 registers: 40 warps per SM hide the gather latency
   using Base = Body;

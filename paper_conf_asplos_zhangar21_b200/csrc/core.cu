@@ -457,6 +457,9 @@ vf_status vf_set_tuning(const char* key, int value) {
   } else if (!strcmp(key, "cluster")) {
     if (value < 0 || value > 1) return VF_ERR_INVALID;
     tuning().cluster = value;
+  } else if (!strcmp(key, "gsort")) {
+    if (value < -1 || value > 1) return VF_ERR_INVALID;
+    tuning().gsort = value;
   } else if (!strcmp(key, "ray_rays")) {
     if (value != 2 && value != 4) return VF_ERR_INVALID;
     tuning().ray_rays = value;
@@ -508,6 +511,18 @@ vf_status vf_create(const vf_config* cfg, vf_ctx** out) {
     size_t g = 0;
     if (d.granularity(&g, &prop, CU_MEM_ALLOC_GRANULARITY_RECOMMENDED) == CUDA_SUCCESS && g)
       c->gran = g;
+  }
+  // Stream-ordered scratch (cudaMallocAsync: batched allocation, the grid-level
+  // type sort) comes from the device's default pool; keep what it has mapped
+  // instead of returning it at every synchronisation (threshold 0 would make
+  // each dispatch re-map its scratch).
+  {
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, c->cfg.device) == cudaSuccess) {
+      uint64_t keep = ~0ull;
+      cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep);
+    }
+    cudaGetLastError();
   }
   // Device heap for the CUDA baseline. The limit can only grow
   // before the first device-malloc kernel of the process; failure here is

@@ -1062,10 +1062,29 @@ struct Lean<A, std::void_t<decltype(A::kLean)>> {
   static constexpr bool value = A::kLean;
 };
 
+constexpr uint32_t kGsChunk = 4096;  // entries per histogram chunk of the grid-level type sort
+// Apps whose heavy methods default to the grid-level type sort (App::kGridSort)
+template <class A, class = void>
+struct GridSortDefault {
+  static constexpr bool value = false;
+};
+template <class A>
+struct GridSortDefault<A, std::void_t<decltype(A::kGridSort)>> {
+  static constexpr bool value = A::kGridSort;
+};
+template <class App, int M, class R>
+cudaError_t launch_gsorted(const uint64_t* objs, uint64_t n, const ArgBlob& args, const DevTable& tbl,
+                           cudaStream_t s);
+
 template <class App, int M, class R>
 cudaError_t launch_grouped_tuned(const uint64_t* objs, uint64_t n, const ArgBlob& args,
                                  const DevTable& tbl, cudaStream_t s) {
   const Tuning& tu = tuning();
+  if constexpr (App::kTypes > 1 && ((HeavyMaskOf<App>::value >> M) & 1u) != 0) {
+    // heavy methods: the whole dispatch list sorted by type (tuning "gsort")
+    const bool gs = tu.gsort >= 0 ? tu.gsort != 0 : GridSortDefault<App>::value;
+    if (gs && tu.regroup != 0 && n >= 2 * kGsChunk) return launch_gsorted<App, M, R>(objs, n, args, tbl, s);
+  }
   if constexpr (Lean<App>::value) {
     if (App::kTypes > 1 && tu.regroup != 0)
       return launch_sorted<App, M, R, App::kUnrollSorted, App::kPrefetch>(objs, n, args, tbl, s);
@@ -1088,6 +1107,172 @@ cudaError_t launch_grouped_tuned(const uint64_t* objs, uint64_t n, const ArgBlob
   if (u == 2) return launch_grouped_pf<App, M, R, 2>(pf, objs, n, args, tbl, s);
   return launch_grouped_pf<App, M, R, 1>(pf, objs, n, args, tbl, s);
   }
+}
+
+// ---------------------------------------------------------------------------
+// Grid-level type sort for heavy methods (tuning key "gsort"; App::kHeavyMask).
+//
+// A CTA-level sort still leaves the warps that straddle two type runs of its
+// tile running a long body twice (once per type, half the lanes each), and
+// heavy bodies make every CTA wait for those warps. Because the type comes
+// from the pointer alone (COAL / TypePointer), the whole dispatch list can be
+// counting-sorted by type first — (pointer, index) pairs, index order kept
+// within a type — so only the warps at the <= T-1 run boundaries of the whole
+// list are mixed. Three small passes (per-chunk type histogram, per-type scan,
+// placement) move 8 B in and 12 B out per entry; then one thread per sorted
+// entry resolves its pointer again and runs the grouped direct call with the
+// entry's ORIGINAL index (bodies that use it, e.g. graph work-entry chunks,
+// see the same index). Calls are order-independent (reading G8).
+// ---------------------------------------------------------------------------
+
+template <class App, class R>
+__device__ __forceinline__ uint32_t gs_type(const unsigned char* smem, const DevTable& tbl, uint64_t p) {
+  if (!p) return 0xFFFFu;
+  uint64_t a;
+  uint32_t hint = 0;
+  uint32_t t = R::resolve(smem, tbl, p, a, hint);
+  if (t >= (uint32_t)App::kTypes) t = type_from_vptr<App>(a, tbl);  // fallback
+  return t < (uint32_t)App::kTypes ? t : 0xFFFFu;                 // unresolvable: dropped (as the dispatch would)
+}
+
+template <class App, class R>
+__global__ void __launch_bounds__(256) k_gs_hist(const uint64_t* __restrict__ objs, uint64_t n, DevTable tbl,
+                                                 uint32_t* __restrict__ hist) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  __shared__ uint32_t h[32];
+  if constexpr (R::kNeedsTable) R::stage(smem, tbl);
+  if (threadIdx.x < 32) h[threadIdx.x] = 0;
+  __syncthreads();
+  const uint64_t base = (uint64_t)blockIdx.x * kGsChunk;
+  const uint32_t lane = threadIdx.x & 31u;
+  for (uint32_t r = 0; r < kGsChunk / 256; ++r) {
+    const uint64_t i = base + (uint64_t)r * 256 + threadIdx.x;
+    const uint32_t t = i < n ? gs_type<App, R>(smem, tbl, ldg_u64(objs + i)) : 0xFFFFu;
+    const uint32_t peers = __match_any_sync(0xffffffffu, t);
+    if (t < 32u && lane == (uint32_t)(__ffs(peers) - 1)) atomicAdd(&h[t], (uint32_t)__popc(peers));
+  }
+  __syncthreads();
+  if (threadIdx.x < 32) hist[(uint64_t)blockIdx.x * 32 + threadIdx.x] = h[threadIdx.x];
+}
+
+template <class App, class R>
+__global__ void __launch_bounds__(256) k_gs_place(const uint64_t* __restrict__ objs, uint64_t n, DevTable tbl,
+                                                  const uint32_t* __restrict__ hist,
+                                                  const unsigned long long* __restrict__ totals,
+                                                  uint64_t* __restrict__ sp, uint32_t* __restrict__ si) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  constexpr int kWarps = 256 / 32;
+  __shared__ uint32_t run[32];
+  __shared__ uint32_t wcnt[kWarps][32];
+  __shared__ unsigned long long boff[32];
+  if constexpr (R::kNeedsTable) R::stage(smem, tbl);
+  const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
+  if (threadIdx.x < 32) {
+    // this chunk's first slot of type t = (objects of types < t) + (type t in earlier chunks)
+    const unsigned long long tot = lane < (uint32_t)App::kTypes ? totals[lane] : 0ull;
+    unsigned long long x = tot;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const unsigned long long y = __shfl_up_sync(0xffffffffu, x, o);
+      if (lane >= (uint32_t)o) x += y;
+    }
+    run[lane] = 0;
+    boff[lane] = x - tot + hist[(uint64_t)blockIdx.x * 32 + lane];
+  }
+  const uint64_t base = (uint64_t)blockIdx.x * kGsChunk;
+  for (uint32_t r = 0; r < kGsChunk / 256; ++r) {
+    const uint64_t i = base + (uint64_t)r * 256 + threadIdx.x;
+    const uint64_t p = i < n ? ldg_u64(objs + i) : 0ull;
+    const uint32_t t = i < n ? gs_type<App, R>(smem, tbl, p) : 0xFFFFu;
+    wcnt[warp][lane] = 0;
+    __syncwarp();
+    const uint32_t peers = __match_any_sync(0xffffffffu, t);
+    const uint32_t within = __popc(peers & ((1u << lane) - 1u));
+    if (t < 32u && lane == (uint32_t)(__ffs(peers) - 1)) wcnt[warp][t] = __popc(peers);
+    __syncthreads();
+    if (t < 32u) {
+      uint32_t before = run[t];
+      for (uint32_t w = 0; w < warp; ++w) before += wcnt[w][t];
+      const unsigned long long pos = boff[t] + before + within;
+      sp[pos] = p;
+      si[pos] = (uint32_t)i;
+    }
+    __syncthreads();
+    if (threadIdx.x < 32) {
+      uint32_t c = 0;
+      for (int w = 0; w < kWarps; ++w) c += wcnt[w][threadIdx.x];
+      run[threadIdx.x] += c;
+    }
+    __syncthreads();
+  }
+}
+
+// one thread per type-sorted entry; warps are type-uniform except at run boundaries
+template <class App, int M, class R>
+__global__ void __launch_bounds__(kBlock, MinBlocks<App>::value) k_dispatch_list(
+    const uint64_t* __restrict__ sp, const uint32_t* __restrict__ si, const unsigned long long* __restrict__ totals,
+    ArgBlob args, DevTable tbl) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  __shared__ unsigned long long s_m;
+  if constexpr (R::kNeedsTable) R::stage(smem, tbl);
+  if (threadIdx.x < 32) {
+    // sorted entries = typed objects (nulls and untypable pointers were dropped)
+    unsigned long long x = threadIdx.x < (uint32_t)App::kTypes ? totals[threadIdx.x] : 0ull;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
+    if (threadIdx.x == 0) s_m = x;
+  }
+  __syncthreads();
+  const uint64_t m = s_m;
+  const uint64_t k = (uint64_t)blockIdx.x * kBlock + threadIdx.x;
+  uint64_t p = 0, a = 0, i = 0;
+  uint32_t t = kNF, hint = 0;
+  if (k < m) {
+    p = ldg_u64(sp + k);
+    i = __ldg(si + k);
+    t = R::resolve(smem, tbl, p, a, hint);
+  }
+  group_call<App, M>(t, a, p, i, args, tbl);
+}
+
+uint64_t rank_chunks(uint64_t n);
+cudaError_t scan_type_hist(uint32_t* hist, uint64_t nchunks, uint32_t ntypes, unsigned long long* totals,
+                           cudaStream_t s);
+
+template <class App, int M, class R>
+cudaError_t launch_gsorted(const uint64_t* objs, uint64_t n, const ArgBlob& args, const DevTable& tbl,
+                           cudaStream_t s) {
+  static_assert(App::kTypes <= 32, "one warp scans the type totals");
+  const uint64_t nch = (n + kGsChunk - 1) / kGsChunk;
+  if (nch > 0x7FFFFFFFull || n > 0xFFFFFFFFull) return cudaErrorInvalidValue;
+  const size_t hist_b = 128ull * nch, tot_b = 8ull * 32;
+  const size_t sp_b = 8ull * n, si_b = 4ull * n;
+  unsigned char* scratch = nullptr;
+  cudaError_t e = cudaMallocAsync(reinterpret_cast<void**>(&scratch), hist_b + tot_b + sp_b + si_b + 64, s);
+  if (e != cudaSuccess) return e;
+  uint32_t* hist = reinterpret_cast<uint32_t*>(scratch);
+  unsigned long long* totals = reinterpret_cast<unsigned long long*>(scratch + hist_b);
+  uint64_t* sp = reinterpret_cast<uint64_t*>(scratch + align16(hist_b + tot_b));
+  uint32_t* si = reinterpret_cast<uint32_t*>(reinterpret_cast<unsigned char*>(sp) + sp_b);
+  const size_t tsm = R::kNeedsTable ? table_smem(tbl) : 0;
+  if (tsm > 32 * 1024) {
+    cudaFuncSetAttribute(k_gs_hist<App, R>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tsm);
+    cudaFuncSetAttribute(k_gs_place<App, R>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tsm);
+  }
+  k_gs_hist<App, R><<<(unsigned)nch, 256, tsm, s>>>(objs, n, tbl, hist);
+  e = scan_type_hist(hist, nch, App::kTypes, totals, s);
+  if (e == cudaSuccess) {
+    k_gs_place<App, R><<<(unsigned)nch, 256, tsm, s>>>(objs, n, tbl, hist, totals, sp, si);
+    note_launch(2);
+    // one thread per entry: n threads cover the (<= n) sorted entries
+    constexpr auto kern = k_dispatch_list<App, M, R>;
+    (void)occupancy<kern>(tsm);  // sets the dynamic smem attribute when needed
+    kern<<<grid_for(n, kBlock, ~0ull), kBlock, tsm, s>>>(sp, si, totals, args, tbl);
+    note_launch();
+    e = cudaGetLastError();
+  }
+  cudaFreeAsync(scratch, s);
+  return e;
 }
 
 template <class App, int M, class R>

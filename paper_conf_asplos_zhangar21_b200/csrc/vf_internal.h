@@ -123,6 +123,8 @@ struct Tuning {
   int persistent = -1; // grouped kernels: 1 persistent grid, 0 one tile per CTA, -1 app default (kHeavyMask)
   int cluster = 0;     // vf_gol_run: 1 one thread-block cluster (state in DSMEM) when the grid fits
   int ray_rays = 4;       // ray kernels: pixels (rays) per thread, 2 or 4
+  int gsort = -1;         // COAL / TypePointer heavy methods: 1 = sort the whole dispatch list by type
+                          // first, 0 = per CTA tile only, -1 = app default (App::kGridSort)
 };
 Tuning& tuning();
 
