@@ -755,7 +755,9 @@ vf_status vf_checksum_i32(const int32_t* vals_dev, uint64_t n, long long* out_de
  * the pointer; (pointer, index) pairs, index order kept within a type; the
  * body still receives the entry's original index), 0 sorts per CTA tile
  * only, -1 (default) = the app's choice (N-body and collision sort the list;
- * the graph methods, measured no faster, do not).
+ * the graph methods, measured no faster, do not); "coal_inline" = the largest
+ * COAL table (rows, 0..8, default 8) tested from the kernel parameters rather
+ * than searched in shared memory.
  * The unroll / prefetch / pipeline knobs apply to config 2's app (micro);
  * the other apps run their default launch configuration.
  * VF_ERR_INVALID for unknown keys / values. */

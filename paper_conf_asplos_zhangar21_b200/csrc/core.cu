@@ -384,8 +384,9 @@ DevTable dev_table(vf_ctx* c, uint32_t app) {
   d.ntypes = app_ops(app)->ntypes;
   d.active_types = 0;
   for (uint64_t k : c->type_count[app]) d.active_types += (k != 0);
+  d.inl = t.K <= kTableInline && (int)t.K <= tuning().coal_inline ? 1u : 0u;
   for (uint32_t j = 0; j < kTableInline; ++j) {
-    const bool v = j < t.K && t.K <= kTableInline;
+    const bool v = j < t.K && t.K <= kTableInline;  // (rows are filled whenever they fit)
     d.in_start[j] = v ? t.rows[j].start : ~0ull;
     d.in_len[j] = v ? t.rows[j].end - t.rows[j].start : 0ull;
     d.in_type[j] = v ? t.rows[j].type_id : VF_NOT_FOUND;
@@ -457,6 +458,9 @@ vf_status vf_set_tuning(const char* key, int value) {
   } else if (!strcmp(key, "cluster")) {
     if (value < 0 || value > 1) return VF_ERR_INVALID;
     tuning().cluster = value;
+  } else if (!strcmp(key, "coal_inline")) {
+    if (value < 0 || value > (int)kTableInline) return VF_ERR_INVALID;
+    tuning().coal_inline = value;
   } else if (!strcmp(key, "gsort")) {
     if (value < -1 || value > 1) return VF_ERR_INVALID;
     tuning().gsort = value;

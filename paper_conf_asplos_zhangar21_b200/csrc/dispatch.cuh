@@ -106,7 +106,7 @@ struct ResolveTP {
 struct ResolveCOAL {
   static constexpr bool kNeedsTable = true;
   __device__ static void stage(unsigned char* smem, const DevTable& t) {
-    if (t.K <= kTableInline) return;  // searched in the parameter bank (CTA-uniform)
+    if (t.inl) return;  // searched in the parameter bank (CTA-uniform)
     uint64_t* s_start = reinterpret_cast<uint64_t*>(smem);
     uint64_t* s_end = s_start + t.P;
     uint32_t* s_type = reinterpret_cast<uint32_t*>(s_end + t.P);
@@ -126,7 +126,7 @@ struct ResolveCOAL {
     a = strip(p);  // a TypePointer-tagged pointer is searched (and dereferenced) by its address
     p = a;
     (void)hint;
-    if (tbl.K <= kTableInline) {
+    if (tbl.inl) {
       // p in [start, end) <=> (p - start) < (end - start), unsigned: one
       // 64-bit subtract and one 64-bit compare per row
       uint32_t t = kNF;

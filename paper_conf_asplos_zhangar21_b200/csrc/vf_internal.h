@@ -34,6 +34,7 @@ struct DevTable {
   const uint64_t* vptr;   // ntypes entries: device vTable* per concrete type
   uint32_t ntypes;
   uint32_t active_types;  // concrete types with live objects (launch heuristics)
+  uint32_t inl;           // 1: COAL tests the inline rows below (K <= min(kTableInline, tuning coal_inline))
   uint64_t in_start[kTableInline];  // rows 0..K-1 when K <= kTableInline
   uint64_t in_len[kTableInline];    // end - start (0 for padding rows)
   uint32_t in_type[kTableInline];
@@ -123,6 +124,7 @@ struct Tuning {
   int persistent = -1; // grouped kernels: 1 persistent grid, 0 one tile per CTA, -1 app default (kHeavyMask)
   int cluster = 0;     // vf_gol_run: 1 one thread-block cluster (state in DSMEM) when the grid fits
   int ray_rays = 4;       // ray kernels: pixels (rays) per thread, 2 or 4
+  int coal_inline = 8;    // COAL: largest table (rows) tested from the kernel parameters (0: always shared memory)
   int gsort = -1;         // COAL / TypePointer heavy methods: 1 = sort the whole dispatch list by type
                           // first, 0 = per CTA tile only, -1 = app default (App::kGridSort)
 };
