@@ -267,7 +267,8 @@ enum {
                               multi-chunk vertex combines with atomicMin: label_out must
                               hold a label >= label_in[v], e.g. the previous-but-one
                               iterate); *changed = 1 if it is below label_in[v]          */
-  VF_GRAPH_PR_CONTRIB = 3, /* chunk 0 only: contrib[v] = deg ? rank_in[v]/deg : 0 (fp64);
+  VF_GRAPH_PR_CONTRIB = 3, /* chunk 0 only: contrib[v] = deg ? rank_in[v]/deg : 0, the
+                              fp64 quotient rounded once to fp32 (DESIGN §2 R-PR32);
                               deg-0 vertices add rank_in[v] to *dangling                 */
   VF_GRAPH_PR_UPDATE = 4,  /* rank_out[v] = (float)(base + d*(sum_{N(v)} contrib +
                               *dangling / Vd)); a multi-chunk vertex writes its chunk sum
@@ -319,7 +320,7 @@ typedef struct {
   const uint32_t* col_dev;
   const float* rank_in_dev;
   float* rank_out_dev;
-  double* contrib_dev;
+  float* contrib_dev;          /* V floats (gathered; summed in fp64 by pr_update) */
   double* dangling_dev;
   double base, d, Vd;
   const uint32_t* chunk_dev;

@@ -105,7 +105,7 @@ struct VertexK final : Vertex {
   __device__ void pr_contrib(vf_graph_pr_args a, uint64_t i) {
     if (nchunks(deg, a.C) > 1 && __ldg(a.chunk_dev + i) != 0) return;  // once per vertex
     const float r = a.rank_in_dev[vid];
-    a.contrib_dev[vid] = deg ? (double)r / (double)deg : 0.0;
+    a.contrib_dev[vid] = deg ? (float)((double)r / (double)deg) : 0.0f;
     if (!deg) {
       // dangling mass: one fp64 atomic per group of lanes that get here together
       // (RMAT graphs have millions of isolated vertices: per-lane atomics on one
@@ -123,7 +123,7 @@ struct VertexK final : Vertex {
     double s;
     if constexpr (U == 1) {
       s = 0.0;
-      for_neighbors<1>(a.col_dev, w.b, w.e, [&](uint32_t u) { s += ld_hint(a.contrib_dev + u, keep); });
+      for_neighbors<1>(a.col_dev, w.b, w.e, [&](uint32_t u) { s += (double)ld_hint(a.contrib_dev + u, keep); });
     } else {
       double acc[U];
 #pragma unroll
@@ -131,9 +131,9 @@ struct VertexK final : Vertex {
       uint64_t k = w.b;
       for (; k + U <= w.e; k += U) {
 #pragma unroll
-        for (int j = 0; j < U; ++j) acc[j] += ld_hint(a.contrib_dev + __ldg(a.col_dev + k + j), keep);
+        for (int j = 0; j < U; ++j) acc[j] += (double)ld_hint(a.contrib_dev + __ldg(a.col_dev + k + j), keep);
       }
-      for (; k < w.e; ++k) acc[0] += ld_hint(a.contrib_dev + __ldg(a.col_dev + k), keep);
+      for (; k < w.e; ++k) acc[0] += (double)ld_hint(a.contrib_dev + __ldg(a.col_dev + k), keep);
       s = 0.0;
 #pragma unroll
       for (int j = 0; j < U; ++j) s += acc[j];

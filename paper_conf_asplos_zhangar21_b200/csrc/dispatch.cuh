@@ -52,6 +52,19 @@ struct MinBlocks<A, std::void_t<decltype(A::kMinBlocks)>> {
   static constexpr int value = A::kMinBlocks;
 };
 
+// CTA size of the grid-sorted list kernel (k_dispatch_list). Apps whose heavy
+// grid is only a few CTAs per SM (N-body: 65,536 bodies = 256 CTAs of 256 on
+// 148 SMs, so 108 SMs run two and 40 run one) set a smaller block so the CTAs
+// spread evenly; the register cap stays that of kBlock x kMinBlocks.
+template <class A, class = void>
+struct ListBlock {
+  static constexpr int value = kBlock;
+};
+template <class A>
+struct ListBlock<A, std::void_t<decltype(A::kListBlock)>> {
+  static constexpr int value = A::kListBlock;
+};
+
 __device__ __forceinline__ uint64_t ldg_u64(const uint64_t* p) {
   uint64_t v;
   asm volatile("ld.global.nc.L1::no_allocate.u64 %0, [%1];" : "=l"(v) : "l"(p));
@@ -1208,8 +1221,8 @@ __global__ void __launch_bounds__(256) k_gs_place(const uint64_t* __restrict__ o
 }
 
 // one thread per type-sorted entry; warps are type-uniform except at run boundaries
-template <class App, int M, class R>
-__global__ void __launch_bounds__(kBlock, MinBlocks<App>::value) k_dispatch_list(
+template <class App, int M, class R, int B = ListBlock<App>::value>
+__global__ void __launch_bounds__(B, MinBlocks<App>::value * (kBlock / B)) k_dispatch_list(
     const uint64_t* __restrict__ sp, const uint32_t* __restrict__ si, const unsigned long long* __restrict__ totals,
     ArgBlob args, DevTable tbl) {
   extern __shared__ __align__(16) unsigned char smem[];
@@ -1224,7 +1237,7 @@ __global__ void __launch_bounds__(kBlock, MinBlocks<App>::value) k_dispatch_list
   }
   __syncthreads();
   const uint64_t m = s_m;
-  const uint64_t k = (uint64_t)blockIdx.x * kBlock + threadIdx.x;
+  const uint64_t k = (uint64_t)blockIdx.x * B + threadIdx.x;
   uint64_t p = 0, a = 0, i = 0;
   uint32_t t = kNF, hint = 0;
   if (k < m) {
@@ -1267,7 +1280,8 @@ cudaError_t launch_gsorted(const uint64_t* objs, uint64_t n, const ArgBlob& args
     // one thread per entry: n threads cover the (<= n) sorted entries
     constexpr auto kern = k_dispatch_list<App, M, R>;
     (void)occupancy<kern>(tsm);  // sets the dynamic smem attribute when needed
-    kern<<<grid_for(n, kBlock, ~0ull), kBlock, tsm, s>>>(sp, si, totals, args, tbl);
+    constexpr int B = ListBlock<App>::value;
+    kern<<<grid_for(n, B, ~0ull), B, tsm, s>>>(sp, si, totals, args, tbl);
     note_launch();
     e = cudaGetLastError();
   }

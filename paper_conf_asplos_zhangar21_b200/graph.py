@@ -118,7 +118,7 @@ class Graph:
         self.changed = torch.zeros(1, dtype=torch.int32, device=dev)
         self._rk = [exchange.BlockArray(dtype=torch.float32, **blk) for _ in range(2)]
         self.rk = [b.view for b in self._rk]
-        self._contrib = exchange.BlockArray(dtype=torch.float64, **blk)
+        self._contrib = exchange.BlockArray(dtype=torch.float32, **blk)  # fp32 shares (DESIGN §2 R-PR32)
         self.contrib = self._contrib.view
         self.dangling = torch.zeros(1, dtype=torch.float64, device=dev)
         self.partial = torch.zeros(max(self.E, 1), dtype=torch.float64, device=dev)

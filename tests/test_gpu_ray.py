@@ -67,3 +67,51 @@ def test_ray_full_frame_sampled_rows(ctx):
         rr, hh, _, _ = oracle.ray_render(W, H, types, P, cam, synth.RAY_ALBEDO, row0=int(row), nrows=1,
                                          threads=oracle.max_threads())
         assert np.array_equal(hh[0], hid[row]) and np.array_equal(rr[0], rgb[row])
+
+
+def _edge_scene():
+    """Shapes that sit on the edges of the hoisted fast path's operand ranges
+    (app_ray.cu hit_rays / fast_domain), mixed into a random scene so tiles
+    hold both: the fast path must give hit_t's results, or flag the tile for
+    the per-operation IEEE re-run."""
+    types, P = synth.ray_scene(700, seed=11)
+    extra = []
+    # tangent sphere: the centre ray (odd W, H: d = (0, 0, -1)) has disc == 0 exactly
+    extra.append((1, [1.0, 0.0, -10.0, 1.0]))
+    # grazing spheres: disc tiny positive / tiny negative for the centre ray
+    extra.append((1, [2.0, 0.0, -20.0, 2.0 * (1 + 2 ** -23)]))
+    extra.append((1, [3.0, 0.0, -30.0, 3.0 * (1 - 2 ** -23)]))
+    # spheres outside the fast domain (|centre| > 2^40): tile re-run
+    extra.append((1, [0.0, 0.0, -3.0e12, 1.0e12]))
+    # triangle in the plane y = 0 (contains the origin): det == 0 for the d.y == 0 row
+    extra.append((3, [-1.0, 0.0, -5.0, 1.0, 0.0, -5.0, 0.0, 0.0, -8.0]))
+    # triangle with huge vertices (outside the fast domain)
+    extra.append((3, [-1e10, -1e10, -1e11, 1e10, -1e10, -1e11, 0.0, 1e10, -1e11]))
+    # rects: p == 0 (t == 0 -> miss), tiny |p| (outside [2^-60, 2^60]), one per axis
+    extra.append((2, [0, 0.0, -1.0, 1.0, -9.0, -1.0]))
+    extra.append((2, [1, 1e-30, -1.0, 1.0, -9.0, -1.0]))
+    extra.append((2, [2, -4.0, -0.5, 0.5, -0.5, 0.5]))
+    extra.append((2, [0, 1e25, -1.0, 1.0, -9.0, -1.0]))
+    # planes: the ground (shape 0) plus h == 0 and a tiny h
+    extra.append((0, [0.0]))
+    extra.append((0, [1e-30]))
+    t2 = np.array([t for t, _ in extra], np.uint32)
+    P2 = np.zeros((len(extra), 12), np.float32)
+    for i, (_, q) in enumerate(extra):
+        P2[i, :len(q)] = q
+    # interleave: the special shapes land in several tiles and runs
+    types = np.concatenate([types[:300], t2[:6], types[300:], t2[6:]])
+    P = np.concatenate([P[:300], P2[:6], P[300:], P2[6:]])
+    return types, P
+
+
+@pytest.mark.parametrize("variant", VARIANTS)
+@pytest.mark.parametrize("W,H", [(65, 37), (33, 17)])
+def test_ray_fast_path_edges(ctx, variant, W, H):
+    types, P = _edge_scene()
+    cam = synth.ray_camera(W, H)
+    rgb_ref, hid_ref, _, _ = oracle.ray_render(W, H, types, P, cam, synth.RAY_ALBEDO, threads=oracle.max_threads())
+    r = Ray(ctx, types, P, variant)
+    rgb, hid = r.render(W, H, cam)
+    assert np.array_equal(hid.cpu().numpy(), hid_ref)
+    assert np.array_equal(rgb.cpu().numpy(), rgb_ref)
