@@ -3,8 +3,9 @@
 // vertices on a synthetic RMAT graph, reading G22). Vertex classes by degree
 // bucket: Leaf (deg <= 1), Low (2..15), Mid (16..255), Hub (>= 256). All four
 // implement the same semantics (the oracle's plain loops); each picks the
-// loop shape that suits its degree: Leaf has no loop, Low a plain loop, Mid
-// and Hub unrolled loops with independent accumulators (more loads in flight).
+// loop shape that suits its degree: U independent neighbour ids per step (16 B
+// vector loads of the row, for_edges_v) and U independent accumulators, U = 4
+// for Leaf / Low, 8 for Mid / Hub.
 // High-degree vertices are split into work entries of <= C edges (vf.h), so no
 // lane walks a hub's whole row. (Measured on B200: sharing one member's row
 // across the group's lanes in turn — coalesced but serial per vertex — was
@@ -38,13 +39,13 @@ struct Vertex {
 
 template <int KIND>
 struct VertexK final : Vertex {
-  static constexpr int U = KIND == 0 ? 1 : KIND == 1 ? 1 : KIND == 2 ? 4 : 8;
+  static constexpr int U = KIND <= 1 ? 4 : 8;
   __device__ explicit VertexK(const void* arg) : Vertex(arg) {}
 
   __device__ void bfs_expand(vf_graph_bfs_args a, uint64_t i) {
     const Work w = work_of(a.offs_dev, a.chunk_dev, i, vid, deg, a.C);
     const uint64_t keep = l2_keep();
-    for_neighbors<U>(a.col_dev, w.b, w.e, [&](uint32_t u) {
+    for_edges_v<U>(a.col_dev, w.b, w.e, [&](int, uint32_t u) {
       if (ld_hint_rw(a.depth_dev + u, keep) == -1 && atomicCAS(a.depth_dev + u, -1, a.level + 1) == -1) enqueue(a, u);
     });
   }
@@ -82,22 +83,14 @@ struct VertexK final : Vertex {
     const Work w = work_of(a.offs_dev, a.chunk_dev, i, vid, deg, a.C);
     const uint32_t own = __ldg(a.label_in_dev + vid);
     const uint64_t keep = l2_keep();
+    uint32_t acc[U];
+#pragma unroll
+    for (int j = 0; j < U; ++j) acc[j] = own;
+    for_edges_v<U>(a.col_dev, w.b, w.e,
+                   [&](int j, uint32_t u) { acc[j] = min(acc[j], ld_hint(a.label_in_dev + u, keep)); });
     uint32_t m = own;
-    if constexpr (U == 1) {
-      for_neighbors<1>(a.col_dev, w.b, w.e, [&](uint32_t u) { m = min(m, ld_hint(a.label_in_dev + u, keep)); });
-    } else {
-      uint32_t acc[U];
 #pragma unroll
-      for (int j = 0; j < U; ++j) acc[j] = own;
-      uint64_t k = w.b;
-      for (; k + U <= w.e; k += U) {
-#pragma unroll
-        for (int j = 0; j < U; ++j) acc[j] = min(acc[j], ld_hint(a.label_in_dev + __ldg(a.col_dev + k + j), keep));
-      }
-      for (; k < w.e; ++k) acc[0] = min(acc[0], ld_hint(a.label_in_dev + __ldg(a.col_dev + k), keep));
-#pragma unroll
-      for (int j = 0; j < U; ++j) m = min(m, acc[j]);
-    }
+    for (int j = 0; j < U; ++j) m = min(m, acc[j]);
     if (w.nch == 1) a.label_out_dev[vid] = m;
     else atomicMin(a.label_out_dev + vid, m);
     if (m != own) a.changed_dev[0] = 1u;
@@ -120,24 +113,10 @@ struct VertexK final : Vertex {
   __device__ void pr_update(vf_graph_pr_args a, uint64_t i) {
     const Work w = work_of(a.offs_dev, a.chunk_dev, i, vid, deg, a.C);
     const uint64_t keep = l2_keep();
-    double s;
-    if constexpr (U == 1) {
-      s = 0.0;
-      for_neighbors<1>(a.col_dev, w.b, w.e, [&](uint32_t u) { s += (double)ld_hint(a.contrib_dev + u, keep); });
-    } else {
-      double acc[U];
-#pragma unroll
-      for (int j = 0; j < U; ++j) acc[j] = 0.0;
-      uint64_t k = w.b;
-      for (; k + U <= w.e; k += U) {
-#pragma unroll
-        for (int j = 0; j < U; ++j) acc[j] += (double)ld_hint(a.contrib_dev + __ldg(a.col_dev + k + j), keep);
-      }
-      for (; k < w.e; ++k) acc[0] += (double)ld_hint(a.contrib_dev + __ldg(a.col_dev + k), keep);
-      s = 0.0;
-#pragma unroll
-      for (int j = 0; j < U; ++j) s += acc[j];
-    }
+    double acc[4] = {0.0, 0.0, 0.0, 0.0};  // U gathers in flight, 4 fp64 chains (64 registers)
+    for_edges_v<U>(a.col_dev, w.b, w.e,
+                   [&](int j, uint32_t u) { acc[j & 3] += (double)ld_hint(a.contrib_dev + u, keep); });
+    double s = (acc[0] + acc[1]) + (acc[2] + acc[3]);
     if (w.nch > 1) {
       // last-finisher combine, in chunk order (deterministic)
       a.partial_dev[i] = s;
@@ -163,7 +142,7 @@ struct App {
   static constexpr int kPrefetch = 2;
   static constexpr bool kLean = true;  // default launch configuration only (knob sweeps: micro)
   static constexpr uint32_t kHeavyMask = 0x3Fu;  // one tile per CTA (dispatch.cuh grid_cap)
-  static constexpr int kMinBlocks = 4;           // <= 64 registers: random gathers need resident warps
+  static constexpr int kMinBlocks = 5;           // <= 48 registers: random gathers need resident warps
   using Base = Vertex;
   template <int K>
   using Type = VertexK<K>;

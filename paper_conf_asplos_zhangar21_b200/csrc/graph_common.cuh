@@ -67,6 +67,62 @@ __device__ __forceinline__ void for_neighbors(const uint32_t* __restrict__ col, 
   for (; k < e; ++k) f(__ldg(col + k));
 }
 
+// Visit col[b..e) with f(j, u): the 16 B-aligned middle with 16 B vector
+// loads, U neighbour ids per step (U / 4 loads in flight, then U independent
+// bodies, f's j = 0..U-1 a compile-time lane of independent work after
+// unrolling), the unaligned head and the tail one id at a time with j = 0.
+// (Per-lane 4 B loads cost one L1 wavefront each: RMAT-24 PageRank was bound
+// by L1 throughput, 75% of peak, with half of the wavefronts on `col`.)
+template <int U, class F>
+__device__ __forceinline__ void for_edges_v(const uint32_t* __restrict__ col, uint64_t b, uint64_t e, F&& f) {
+  static_assert(U % 4 == 0, "U is a multiple of 4");
+  uint64_t k = b;
+  uint64_t h = b + ((4u - (uint32_t)((reinterpret_cast<uintptr_t>(col + b) >> 2) & 3u)) & 3u);
+  if (h > e) h = e;
+  for (; k < h; ++k) f(0, __ldg(col + k));
+  for (; k + U <= e; k += U) {
+    uint4 v[U / 4];
+#pragma unroll
+    for (int j = 0; j < U / 4; ++j) v[j] = __ldg(reinterpret_cast<const uint4*>(col + k) + j);
+#pragma unroll
+    for (int j = 0; j < U / 4; ++j) {
+      f(4 * j, v[j].x);
+      f(4 * j + 1, v[j].y);
+      f(4 * j + 2, v[j].z);
+      f(4 * j + 3, v[j].w);
+    }
+  }
+  if (k + 4 <= e && U > 4) {
+    const uint4 v = __ldg(reinterpret_cast<const uint4*>(col + k));
+    f(0, v.x);
+    f(1, v.y);
+    f(2, v.z);
+    f(3, v.w);
+    k += 4;
+  }
+  for (; k < e; ++k) f(0, __ldg(col + k));
+}
+
+// Is there a neighbour u in col[b..e) with pred(u)? 4 ids per 16 B vector
+// load and their 4 predicate loads in flight; stops after the first step
+// that holds a hit (bottom-up BFS: the answer, not the neighbour, matters).
+template <class P>
+__device__ __forceinline__ bool any_edge_v(const uint32_t* __restrict__ col, uint64_t b, uint64_t e, P&& pred) {
+  uint64_t k = b;
+  uint64_t h = b + ((4u - (uint32_t)((reinterpret_cast<uintptr_t>(col + b) >> 2) & 3u)) & 3u);
+  if (h > e) h = e;
+  for (; k < h; ++k)
+    if (pred(__ldg(col + k))) return true;
+  for (; k + 4 <= e; k += 4) {
+    const uint4 v = __ldg(reinterpret_cast<const uint4*>(col + k));
+    const bool p0 = pred(v.x), p1 = pred(v.y), p2 = pred(v.z), p3 = pred(v.w);
+    if (p0 | p1 | p2 | p3) return true;
+  }
+  for (; k < e; ++k)
+    if (pred(__ldg(col + k))) return true;
+  return false;
+}
+
 __device__ __forceinline__ uint32_t nchunks(uint32_t deg, uint32_t C) { return deg <= C ? 1u : (deg + C - 1) / C; }
 
 // The edge range of work entry i of vertex (vid, deg): chunk c of <= C edges.
