@@ -467,6 +467,9 @@ vf_status vf_set_tuning(const char* key, int value) {
   } else if (!strcmp(key, "ray_rays")) {
     if (value != 2 && value != 4) return VF_ERR_INVALID;
     tuning().ray_rays = value;
+  } else if (!strcmp(key, "ray_parts")) {
+    if (value != -1 && (value < 1 || value > 16)) return VF_ERR_INVALID;
+    tuning().ray_parts = value;
   } else {
     return VF_ERR_INVALID;
   }

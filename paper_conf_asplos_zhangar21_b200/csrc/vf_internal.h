@@ -124,6 +124,7 @@ struct Tuning {
   int persistent = -1; // grouped kernels: 1 persistent grid, 0 one tile per CTA, -1 app default (kHeavyMask)
   int cluster = 0;     // vf_gol_run: 1 one thread-block cluster (state in DSMEM) when the grid fits
   int ray_rays = 4;       // ray kernels: pixels (rays) per thread, 2 or 4
+  int ray_parts = -1;     // ray COAL / TypePointer: shape parts per pixel block (1..16; -1: balance the last wave)
   int coal_inline = 8;    // COAL: largest table (rows) tested from the kernel parameters (0: always shared memory)
   int gsort = -1;         // COAL / TypePointer heavy methods: 1 = sort the whole dispatch list by type
                           // first, 0 = per CTA tile only, -1 = app default (App::kGridSort)

@@ -115,3 +115,22 @@ def test_ray_fast_path_edges(ctx, variant, W, H):
     rgb, hid = r.render(W, H, cam)
     assert np.array_equal(hid.cpu().numpy(), hid_ref)
     assert np.array_equal(rgb.cpu().numpy(), rgb_ref)
+
+
+@pytest.mark.parametrize("variant", ["coal", "typeptr"])
+@pytest.mark.parametrize("parts", [1, 3, 16])
+def test_ray_shape_parts(ctx, variant, parts):
+    """The direct kernel over 1 / 3 / 16 shape parts (in-kernel shading vs
+    atomicMin of the keys + k_ray_shade) gives the oracle's frame."""
+    W, H, S = 200, 120, 2600
+    types, P = synth.ray_scene(S, seed=5)
+    cam = synth.ray_camera(W, H)
+    rgb_ref, hid_ref, _, _ = oracle.ray_render(W, H, types, P, cam, synth.RAY_ALBEDO, threads=oracle.max_threads())
+    r = Ray(ctx, types, P, variant)
+    vf.set_tuning("ray_parts", parts)
+    try:
+        rgb, hid = r.render(W, H, cam)
+    finally:
+        vf.set_tuning("ray_parts", -1)
+    assert np.array_equal(hid.cpu().numpy(), hid_ref)
+    assert np.array_equal(rgb.cpu().numpy(), rgb_ref)
