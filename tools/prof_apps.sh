@@ -12,7 +12,7 @@ cap() {  # name app variant kernel-regex [skip]
 }
 kern() {  # app -> kernel regex of its dominant dispatch
   case $1 in
-    ray) echo "regex:k_ray_";;
+    ray) echo "regex:k_ray_(direct|virtual)";;
     gen) echo "regex:k_step_.*gen::";;
     gol) echo "regex:k_step_.*gol::";;
     traf) echo "regex:traf::App, \(int\)1";;
