@@ -10,6 +10,16 @@ Multi-GPU (``rank``/``world``): vertex ids are split into contiguous blocks;
 each rank dispatches only its owned vertices and the per-iteration state
 (depth / labels / contributions) is exchanged with an all-gather over the
 process group (NCCL on B200, gloo on CPU tests).
+
+State layout (hot-first): the per-vertex state arrays and the CSR the bodies
+read are indexed by a STORAGE slot, not by the vertex id: within each rank's
+block, slots are assigned by descending degree (ties by id), so the state of
+the hubs that most rows gather (RMAT: the >= 256-degree class holds ~70% of
+the arcs) sits in a few dense lines at the start of the block. The vertex
+objects, their allocation and the dispatch order stay in vertex-id order (the
+recipe's random permutation: types interleaved); each object's `vid` field is
+its storage slot. Rows keep their CSR order (same summation order), labels
+are original vertex ids, and every result is returned indexed by vertex id.
 """
 from __future__ import annotations
 
@@ -69,6 +79,28 @@ def work_entries(deg: np.ndarray, lo: int, hi: int, C: int):
     return vid, chunk
 
 
+def _csr_by_slot(offs: np.ndarray, col: np.ndarray, perm, inv, dev):
+    """The CSR in storage-slot space: row s is vertex inv[s]'s row, in the same
+    order, with every neighbour id replaced by its slot (setup, on the GPU)."""
+    offs_t = torch.from_numpy(np.ascontiguousarray(offs, dtype=np.int64)).to(dev)
+    col_t = torch.from_numpy(np.ascontiguousarray(col, dtype=np.uint32).view(np.int32)).to(dev)
+    V, E = len(offs) - 1, len(col)
+    deg_s = (offs_t[1:] - offs_t[:-1])[inv]
+    offs_s = torch.zeros(V + 1, dtype=torch.int64, device=dev)
+    torch.cumsum(deg_s, 0, out=offs_s[1:])
+    col_s = torch.empty(E, dtype=torch.int32, device=dev)
+    step = 1 << 26  # arcs per pass (bounded temporaries)
+    if E:
+        row = torch.repeat_interleave(torch.arange(V, device=dev), deg_s)
+        for k0 in range(0, E, step):
+            k1 = min(E, k0 + step)
+            r = row[k0:k1]
+            src = offs_t[inv[r]] + (torch.arange(k0, k1, device=dev) - offs_s[r])
+            col_s[k0:k1] = perm[col_t[src].long()].int()
+        del row
+    return offs_s, col_s
+
+
 class Graph:
     def __init__(self, ctx: vf.Ctx, offs: np.ndarray, col: np.ndarray, variant: str = "typeptr",
                  rank: int = 0, world: int = 1, group=None, chunk: int = 256):
@@ -82,24 +114,33 @@ class Graph:
         self.rank, self.world, self.group = rank, world, group
         # owned vertex block [lo, hi)
         self.lo, self.hi, self.per = block_range(V, rank, world)
-        self.offs = torch.from_numpy(np.ascontiguousarray(offs, dtype=np.uint64).view(np.int64)).to(dev)
-        self.col = torch.from_numpy(np.ascontiguousarray(col, dtype=np.uint32).view(np.int32)).to(dev)
         deg = np.diff(np.asarray(offs, dtype=np.int64))
+        # storage slot of every vertex (hot-first within each rank's block)
+        perm = np.empty(V, np.int64)
+        for r in range(world):
+            blo, bhi, _ = block_range(V, r, world)
+            order = np.argsort(-deg[blo:bhi], kind="stable")
+            perm[blo + order] = np.arange(blo, bhi, dtype=np.int64)
+        self.perm = torch.from_numpy(perm).to(dev)        # vertex id -> slot
+        self.inv = torch.empty_like(self.perm)
+        self.inv[self.perm] = torch.arange(V, dtype=torch.int64, device=dev)  # slot -> vertex id
+        self.offs, self.col = _csr_by_slot(offs, col, self.perm, self.inv, dev)
         types = synth.vertex_types(offs)
         self.types_np = types
         own = np.arange(self.lo, self.hi)
-        ctor = np.stack([own.astype(np.uint32), deg[own].astype(np.uint32)], axis=1).copy()
+        ctor = np.stack([perm[own].astype(np.uint32), deg[own].astype(np.uint32)], axis=1).copy()
         ctor_t = torch.from_numpy(ctor.view(np.int32)).to(dev)
         tt = torch.from_numpy(types[own].astype(np.int32)).to(dev)
         objs = ctx.alloc_for(variant, vf.APP_GRAPH, tt, ctor_t)
-        # vobj is indexed by global vertex id; only the owned block is filled on this rank
+        # the owned objects in vertex-id order; vobj is indexed by storage slot
+        # (BFS appends a discovered slot's entries); only the owned block is filled
+        self.owned = objs
         self.vobj = torch.zeros(V, dtype=torch.int64, device=dev)
-        self.vobj[self.lo:self.hi] = objs
-        self.owned = self.vobj[self.lo:self.hi]
-        # work entries of the owned block (one virtual call each)
+        self.vobj[self.perm[self.lo:self.hi]] = objs
+        # work entries of the owned block in vertex-id order (one virtual call each)
         evid, ech = work_entries(deg, self.lo, self.hi, self.C)
         self.E = len(evid)
-        self.entries = self.vobj[torch.from_numpy(evid).to(dev)].contiguous()
+        self.entries = objs[torch.from_numpy(evid - self.lo).to(dev)].contiguous()
         self.entry_chunk = torch.from_numpy(ech.view(np.int32)).to(dev)
         e_all = int(np.maximum(1, (deg + self.C - 1) // self.C).sum())
         # per-vertex state in persistent buffers padded to per * world rows; the
@@ -127,6 +168,10 @@ class Graph:
         torch.cuda.synchronize(dev)
 
     # ---------------------------------------------------------------- helpers
+    def by_id(self, t):
+        """A per-slot state array re-indexed by vertex id."""
+        return t[self.perm]
+
     def _allreduce_sum(self, t, stream=None):
         exchange.allreduce_(t, self.world, self.group, stream)
 
@@ -144,6 +189,7 @@ class Graph:
         bits (and every mode at world > 1): one virtual bfs_probe_bits() per owned work entry per
         level over a frontier bitmap whose owned slices are all-gathered (multi-GPU)."""
         L = vf.lib()
+        src_id, src = src, int(self.perm[src].item())  # its storage slot
         st = L.vf_graph_bfs_init(self.V, self.depth.data_ptr(), src, self.vobj.data_ptr(), self.offs.data_ptr(),
                                  self.C, self.q[0].data_ptr(), self.qc[0].data_ptr(), self.count.data_ptr(),
                                  vf._stream(None))
@@ -202,7 +248,7 @@ class Graph:
         else:
             level, calls = self._bfs_bits(src)
         self.calls = calls
-        return self.depth, level, calls
+        return self.by_id(self.depth), level, calls
 
     def _bfs_bits(self, src: int):
         """Bottom-up BFS over frontier bitmaps (multi-GPU): per level
@@ -237,9 +283,10 @@ class Graph:
     # ---------------------------------------------------------------- CC
     def cc(self, max_iters: int = 10 ** 6):
         """Jacobi min-label propagation until no label changes; returns (labels, iters, calls)."""
-        L = vf.lib()
-        L.vf_iota_u32(self.V, self.lab[0].data_ptr(), vf._stream(None))
-        L.vf_iota_u32(self.V, self.lab[1].data_ptr(), vf._stream(None))  # >= every later label (atomicMin combine)
+        # initial label of a slot = its vertex id; the other buffer too (>= every
+        # later label: the atomicMin combine of multi-chunk vertices)
+        self.lab[0].copy_(self.inv)
+        self.lab[1].copy_(self.inv)
         it, calls = 0, 0
         while it < max_iters:
             self.changed.zero_()
@@ -255,7 +302,7 @@ class Graph:
             if _sync_scalar(self.changed) == 0:
                 break
         self.calls = calls
-        return self.lab[0], it, calls
+        return self.by_id(self.lab[0]), it, calls
 
     # ---------------------------------------------------------------- PageRank
     def pr_init(self):
@@ -283,4 +330,4 @@ class Graph:
             calls += self.pr_iteration(d)
         self._rk[0].gather()  # ranks stay on their owner during the iterations
         self.calls = calls
-        return self.rk[0], calls
+        return self.by_id(self.rk[0]), calls

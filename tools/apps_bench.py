@@ -421,10 +421,10 @@ def app_graph(env, variants, pk, cpu=True, scale=24, small=False):
         g = Graph(env.ctx, offs, col, v, env.rank, env.world, env.group)
         ms_b = env.timed(lambda: g.bfs(src, mode=bfs_mode), 2, 1)
         calls_b = env.sum_i(g.calls)
-        d = g.depth.cpu().numpy()
+        d = g.by_id(g.depth).cpu().numpy()
         ms_c = env.timed(lambda: g.cc(), 1, 1)
         calls_c = env.sum_i(g.calls)
-        lab = g.lab[0].cpu().numpy()
+        lab = g.by_id(g.lab[0]).cpu().numpy()
         g.pr_init()
         ms_p = env.timed(lambda: g.pr_iteration(), 10, 2)
         calls_p = env.sum_i(2 * g.E)

@@ -47,12 +47,12 @@ def main():
                 vf.set_tuning("gsort", gs)
                 g = Graph(ctx, offs, col, v, chunk=C)
                 ms_b = env.timed(lambda: g.bfs(src), 2, 1)
-                d = g.depth.cpu().numpy()
+                d = g.by_id(g.depth).cpu().numpy()
                 ms_c = env.timed(lambda: g.cc(), 1, 1)
-                lab = g.lab[0].cpu().numpy()
+                lab = g.by_id(g.lab[0]).cpu().numpy()
                 g.pr_init()
                 ms_p = env.timed(lambda: g.pr_iteration(), a.pr_iters, 2)
-                rk = g.rk[0].cpu().numpy().astype(np.float64)
+                rk = g.by_id(g.rk[0]).cpu().numpy().astype(np.float64)
                 ok = True
                 if ref is None:
                     ref = (d, lab, rk)
