@@ -75,3 +75,29 @@ def test_graph_f6_fixture(ctx):
         assert list(depth.cpu().numpy()) == [0, 1, 2, 3, -1, -1]
         label, _, _ = g.cc()
         assert list(label.cpu().numpy()) == [0, 0, 0, 0, 4, 4]
+
+
+@pytest.mark.parametrize("variant", VARIANTS)
+def test_graph_degenerate_graphs(ctx, variant):
+    """No edges (every vertex dangling: PageRank stays uniform), one edge plus
+    isolated vertices, and a star whose centre spans several work entries
+    (chunk 3): BFS / CC exact, PageRank 1e-5, against the oracle; the results
+    come back by vertex id through the hot-first state slots."""
+    star = [(0, k) for k in range(1, 12)]
+    for V, edges, src in ((5, [], 2), (6, [(2, 4)], 2), (14, star, 5)):
+        offs, col = synth.csr_from_edges(V, edges)
+        types = synth.vertex_types(offs)
+        g = Graph(ctx, offs, col, variant, chunk=3)
+        d_ref, lv_ref, _, _ = oracle.graph_bfs(offs, col, types, src)
+        for mode in ("topdown", "bottomup", "hybrid"):
+            depth, levels, _ = g.bfs(src, mode=mode)
+            assert np.array_equal(depth.cpu().numpy(), d_ref), mode
+            assert mode == "bottomup" or levels == lv_ref, mode
+        l_ref, it_ref, _, _ = oracle.graph_cc(offs, col, types)
+        label, iters, _ = g.cc()
+        assert np.array_equal(label.cpu().numpy().view(np.uint32), l_ref) and iters == it_ref
+        r_ref, _ = oracle.graph_pr(offs, col, types, iters=7)
+        rank, _ = g.pagerank(7)
+        np.testing.assert_allclose(rank.cpu().numpy(), r_ref, rtol=1e-5, atol=0)
+        if not edges:
+            np.testing.assert_allclose(r_ref, 1.0 / V, rtol=1e-6)
