@@ -134,3 +134,17 @@ def test_ray_shape_parts(ctx, variant, parts):
         vf.set_tuning("ray_parts", -1)
     assert np.array_equal(hid.cpu().numpy(), hid_ref)
     assert np.array_equal(rgb.cpu().numpy(), rgb_ref)
+
+
+@pytest.mark.parametrize("variant", VARIANTS)
+def test_ray_empty_and_single_shape_scenes(ctx, variant):
+    """No shapes at all (every pixel a miss) and a one-shape scene: the oracle's frame."""
+    W, H = 17, 9
+    cam = synth.ray_camera(W, H)
+    for S in (0, 1):
+        types, P = synth.ray_scene(S, seed=2)
+        rgb_ref, hid_ref, _, _ = oracle.ray_render(W, H, types, P, cam, synth.RAY_ALBEDO)
+        r = Ray(ctx, types, P, variant)
+        rgb, hid = r.render(W, H, cam)
+        assert np.array_equal(hid.cpu().numpy(), hid_ref)
+        assert np.array_equal(rgb.cpu().numpy(), rgb_ref)
