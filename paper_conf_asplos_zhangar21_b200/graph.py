@@ -101,9 +101,31 @@ def _csr_by_slot(offs: np.ndarray, col: np.ndarray, perm, inv, dev):
     return offs_s, col_s
 
 
+HOT_DEGREE = 0  # 0: every vertex by degree (measured best, DESIGN §5 "Graph vertex order")
+
+
+def slot_order(deg: np.ndarray, V: int, world: int, hot_degree: int = HOT_DEGREE) -> np.ndarray:
+    """perm[v] = storage slot of vertex v: within each rank's block, the hot
+    vertices (degree >= hot_degree) first by descending degree (ties by id),
+    then every other vertex in id order — so the cold majority's own state
+    accesses (in dispatch = id order) stay monotone, and the state every row
+    gathers most (the high-degree endpoints) is dense. hot_degree = 0: a full
+    degree sort."""
+    perm = np.empty(V, np.int64)
+    for r in range(world):
+        blo, bhi, _ = block_range(V, r, world)
+        d = deg[blo:bhi]
+        hot = np.flatnonzero(d >= hot_degree)
+        hot = hot[np.argsort(-d[hot], kind="stable")]
+        cold = np.flatnonzero(d < hot_degree)
+        order = np.concatenate([hot, cold])
+        perm[blo + order] = np.arange(blo, bhi, dtype=np.int64)
+    return perm
+
+
 class Graph:
     def __init__(self, ctx: vf.Ctx, offs: np.ndarray, col: np.ndarray, variant: str = "typeptr",
-                 rank: int = 0, world: int = 1, group=None, chunk: int = 256):
+                 rank: int = 0, world: int = 1, group=None, chunk: int = 256, hot_degree: int = HOT_DEGREE):
         self.ctx, self.variant = ctx, variant
         self.v = vf.VARIANTS[variant]
         dev = torch.device(f"cuda:{ctx.device}")
@@ -116,11 +138,7 @@ class Graph:
         self.lo, self.hi, self.per = block_range(V, rank, world)
         deg = np.diff(np.asarray(offs, dtype=np.int64))
         # storage slot of every vertex (hot-first within each rank's block)
-        perm = np.empty(V, np.int64)
-        for r in range(world):
-            blo, bhi, _ = block_range(V, r, world)
-            order = np.argsort(-deg[blo:bhi], kind="stable")
-            perm[blo + order] = np.arange(blo, bhi, dtype=np.int64)
+        perm = slot_order(deg, V, world, hot_degree)
         self.perm = torch.from_numpy(perm).to(dev)        # vertex id -> slot
         self.inv = torch.empty_like(self.perm)
         self.inv[self.perm] = torch.arange(V, dtype=torch.int64, device=dev)  # slot -> vertex id

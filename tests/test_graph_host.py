@@ -14,13 +14,24 @@ import synth
 from paper_conf_asplos_zhangar21_b200 import graph as G
 
 
-def _perm(deg, V, world):
+def _perm(deg, V, world, hot=0):
+    """Brute force of the slot definition: per block, vertices of degree >=
+    hot by descending degree (ties by id), then the rest by id."""
     perm = np.empty(V, np.int64)
     for r in range(world):
         lo, hi, _ = G.block_range(V, r, world)
-        order = np.argsort(-deg[lo:hi], kind="stable")
-        perm[lo + order] = np.arange(lo, hi)
+        key = sorted(range(lo, hi), key=lambda v: (0, -deg[v], v) if deg[v] >= hot else (1, 0, v))
+        perm[np.array(key, dtype=np.int64)] = np.arange(lo, hi)
     return perm
+
+
+@pytest.mark.parametrize("hot", [0, 4, 16, 1 << 30])
+@pytest.mark.parametrize("world", [1, 3])
+def test_slot_order_matches_definition(hot, world):
+    offs, col = synth.rmat_graph(10, seed=7)
+    V = len(offs) - 1
+    deg = np.diff(offs.astype(np.int64))
+    assert np.array_equal(G.slot_order(deg, V, world, hot), _perm(deg, V, world, hot))
 
 
 @pytest.mark.parametrize("scale,world", [(8, 1), (10, 1), (10, 3)])

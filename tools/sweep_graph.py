@@ -35,6 +35,7 @@ def main():
     ap.add_argument("--chunks", default="256,64")
     ap.add_argument("--gsort", default="0,1")
     ap.add_argument("--pr-iters", type=int, default=10)
+    ap.add_argument("--hot", default="16", help="hot_degree values (graph.slot_order)")
     a = ap.parse_args()
     ctx = vf.Ctx(0, cuda_heap_bytes=8 << 30)
     env = Env(ctx)
@@ -43,9 +44,9 @@ def main():
     ref = None
     for v in a.variants.split(","):
         for C in [int(x) for x in a.chunks.split(",")]:
-            for gs in [int(x) for x in a.gsort.split(",")]:
+            for gs, hd in [(int(x), int(h)) for x in a.gsort.split(",") for h in a.hot.split(",")]:
                 vf.set_tuning("gsort", gs)
-                g = Graph(ctx, offs, col, v, chunk=C)
+                g = Graph(ctx, offs, col, v, chunk=C, hot_degree=hd)
                 ms_b = env.timed(lambda: g.bfs(src), 2, 1)
                 d = g.by_id(g.depth).cpu().numpy()
                 ms_c = env.timed(lambda: g.cc(), 1, 1)
@@ -59,7 +60,7 @@ def main():
                 else:
                     ok = bool(np.array_equal(ref[0], d) and np.array_equal(ref[1], lab)
                               and np.allclose(rk, ref[2], rtol=1e-5, atol=0))
-                print(json.dumps({"variant": v, "C": C, "gsort": gs, "bfs_ms": ms_b, "cc_ms": ms_c,
+                print(json.dumps({"variant": v, "C": C, "gsort": gs, "hot_degree": hd, "bfs_ms": ms_b, "cc_ms": ms_c,
                                   "pr_iter_ms": ms_p, "agree": ok}), flush=True)
                 del g
                 env.free()
