@@ -207,7 +207,7 @@ class Graph:
         bits (and every mode at world > 1): one virtual bfs_probe_bits() per owned work entry per
         level over a frontier bitmap whose owned slices are all-gathered (multi-GPU)."""
         L = vf.lib()
-        src_id, src = src, int(self.perm[src].item())  # its storage slot
+        src = int(self.perm[src].item())  # the source vertex id -> its storage slot
         st = L.vf_graph_bfs_init(self.V, self.depth.data_ptr(), src, self.vobj.data_ptr(), self.offs.data_ptr(),
                                  self.C, self.q[0].data_ptr(), self.qc[0].data_ptr(), self.count.data_ptr(),
                                  vf._stream(None))
