@@ -1099,6 +1099,14 @@ cudaError_t launch_grouped_tuned(const uint64_t* objs, uint64_t n, const ArgBlob
     if (gs && tu.regroup != 0 && n >= 2 * kGsChunk) return launch_gsorted<App, M, R>(objs, n, args, tbl, s);
   }
   if constexpr (Lean<App>::value) {
+    if constexpr (((HeavyMaskOf<App>::value >> M) & 1u) != 0 && App::kUnrollSorted > 1) {
+      // a small dispatch of a long body (graph: the top-down expansion of the
+      // BFS source's chunks, a few thousand entries) is a grid of a few CTAs:
+      // one entry per thread doubles its parallelism (measured at RMAT-24:
+      // level-0 expansion 1.75 -> 1.0 ms, the CUDA kernel's one-per-thread)
+      if (App::kTypes > 1 && tu.regroup != 0 && n < (uint64_t)num_sms() * kBlock * 4)
+        return launch_sorted<App, M, R, 1, App::kPrefetch>(objs, n, args, tbl, s);
+    }
     if (App::kTypes > 1 && tu.regroup != 0)
       return launch_sorted<App, M, R, App::kUnrollSorted, App::kPrefetch>(objs, n, args, tbl, s);
     return launch_grouped<App, M, R, App::kUnroll, App::kPrefetch>(objs, n, args, tbl, s);

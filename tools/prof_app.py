@@ -52,6 +52,8 @@ def main():
                 g.pr_iteration()
         elif a.app == "graph-cc":
             g.cc(max_iters=a.steps)
+        elif a.app == "graph-bfs-hybrid":
+            g.bfs(src, mode="hybrid")
         else:
             g.bfs(src)
     elif a.app == "stut":
