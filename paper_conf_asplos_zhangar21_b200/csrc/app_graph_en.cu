@@ -277,7 +277,7 @@ struct VertexK final : ChiVertex {
     for (int j = 0; j < U; ++j) m = min(m, acc[j]);
     if (w.nch == 1) a.label_out_dev[vid] = m;
     else atomicMin(a.label_out_dev + vid, m);
-    if (m != own) a.changed_dev[0] = 1u;
+    if (m != own && __ldcg(a.changed_dev) == 0u) a.changed_dev[0] = 1u;  // (see app_graph.cu cc_update)
   }
   __device__ __forceinline__ void pr_init_t(const vf_graph_en_pr_args& a, uint64_t i) {
     if (nchunks(deg, a.C) > 1 && __ldg(a.chunk_dev + i) != 0) return;  // once per vertex

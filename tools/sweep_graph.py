@@ -35,7 +35,7 @@ def main():
     ap.add_argument("--chunks", default="256,64")
     ap.add_argument("--gsort", default="0,1")
     ap.add_argument("--pr-iters", type=int, default=10)
-    ap.add_argument("--hot", default="16", help="hot_degree values (graph.slot_order)")
+    ap.add_argument("--hot", default="0", help="hot_degree values (graph.slot_order)")
     a = ap.parse_args()
     ctx = vf.Ctx(0, cuda_heap_bytes=8 << 30)
     env = Env(ctx)
